@@ -1,0 +1,383 @@
+"""TEST INFRASTRUCTURE ONLY -- reference fusion planner, written step by step
+from the paper (Qiao et al., CGO'19, §II-§III), plus a brute-force optimum.
+
+Only tests/ (and bench.py's diagnostics) may import this module; the product
+planner (paper_conf_cgo_qiaorht19_b200/csrc/planner.cpp) shares no code with it.
+
+Contents, each in the paper's notation:
+  kernel_costs()  nALU / nSFU per kernel (SURVEY O1-d reading: explicit cost, else
+                  an opcode count)
+  edge_weights()  scenario per edge and w_e (Eqs. 3-12)
+  is_legal()      dependence (Fig. 2), resources (Eq. 2,
+                  PAPER.md:296-321), header, profitability
+                    -- readings O1-f/g/h/l
+  stoer_wagner()  global min cut, deterministic tie-breaks O1-j ([14])
+  get_legal_partitions()  Alg. 1
+  brute_force()   exact maximum of Eq. 1 over all partitions into legal blocks
+                  (the paper's "exhaustive search")
+
+Weights are lexicographic pairs (real, eps-count) with the real part in fixed
+point q = floor(w * 2^20 + 0.5) (reading O1-i): sums are exact, so ties
+("the first one encountered") are decided identically here
+and in the C++ planner.
+"""
+from __future__ import annotations
+
+import math
+from dataclasses import dataclass, field
+
+SFU_OPS = {"SQRT", "EXP", "LOG", "POW"}
+NONARITH = {"LOAD", "CONST"}
+FIX = 1 << 20
+
+
+@dataclass
+class Model:
+    """Hardware-model constants."""
+    tg: float = 400.0       # global-memory access, cycles
+    ts: float = 4.0         # shared-memory access, "a few cycles"
+    c_alu: float = 4.0
+    c_sfu: float = 16.0     # not given; reading O1-b
+    gamma: float = 0.0      # omitted in the example
+    c_mshared: float = 2.0
+    phi_mode: int = 0       # 0 = PAPER (per-tap recompute), 1 = STAGED (O1-g B200 profile)
+    tile_w: int = 32
+    tile_h: int = 32
+    eq3_mode: int = 0       # 0: IS*tg/ts as printed; 1: IS*(tg-ts)  (O1-a)
+
+
+PAPER_PROFILE = Model()
+B200_PROFILE = Model(c_mshared=5.0, phi_mode=1)
+
+
+@dataclass
+class Graph:
+    n: int                       # kernels
+    kind: list                   # "point" / "local"
+    inputs: list                 # image ids per kernel
+    n_inputs: int
+    rx: list
+    ry: list
+    mode: list
+    outputs: set
+    bpp: int
+    cost: list                   # (n_alu, n_sfu)
+    edges: list = field(default_factory=list)   # (ks, kd) unique, consumer-major order
+    consumers: list = field(default_factory=list)
+    producers: list = field(default_factory=list)
+
+
+def kernel_costs(o: dict) -> tuple[int, int]:
+    """nALU/nSFU of a kernel: explicit `cost`, else an opcode count (reading O1-d).
+    Local: 2*nnz(mask)-1 multiply-adds plus the post program's ops."""
+    if o.get("cost") is not None:
+        return int(o["cost"][0]), int(o["cost"][1])
+    prog = o["prog"] if o["kind"] == "point" else o["post"]
+    n_sfu = sum(1 for t in prog if t[0] in SFU_OPS)
+    n_alu = sum(1 for t in prog if t[0] not in NONARITH and t[0] not in SFU_OPS)
+    if o["kind"] == "local":
+        nnz = sum(1 for r in o["mask"] for v in r if v != 0.0)
+        n_alu += 2 * max(nnz, 1) - 1
+    return n_alu, n_sfu
+
+
+def graph(spec: dict) -> Graph:
+    ops = spec["ops"]
+    n_in = spec["n_inputs"]
+    g = Graph(n=len(ops), kind=[o["kind"] for o in ops], inputs=[list(o["inputs"]) for o in ops],
+              n_inputs=n_in,
+              rx=[len(o["mask"][0]) // 2 if o["kind"] == "local" else 0 for o in ops],
+              ry=[len(o["mask"]) // 2 if o["kind"] == "local" else 0 for o in ops],
+              mode=[o.get("mode") for o in ops], outputs=set(spec["outputs"]),
+              bpp=4, cost=[kernel_costs(o) for o in ops])
+    g.consumers = [[] for _ in ops]
+    g.producers = [[] for _ in ops]
+    for kd, o in enumerate(ops):
+        for img in o["inputs"]:
+            if img >= n_in:
+                ks = img - n_in
+                if ks not in g.producers[kd]:
+                    g.producers[kd].append(ks)
+                    g.consumers[ks].append(kd)
+                    g.edges.append((ks, kd))
+    return g
+
+
+# ------------------------------------------------------------- legality
+
+
+def _dependence_legal(g: Graph, P: set) -> bool:
+    """Reading O1-f of Fig. 2: one sink; every other kernel has all consumers inside
+    and is not a pipeline output (Fig. 2c); every image a non-source kernel reads
+    from outside P is also read by a source kernel (Fig. 2b legal / 2d illegal)."""
+    sinks = [k for k in P if not any(c in P for c in g.consumers[k])]
+    if len(sinks) != 1:
+        return False
+    for k in P:
+        if k == sinks[0]:
+            continue
+        if (g.n_inputs + k) in g.outputs or any(c not in P for c in g.consumers[k]):
+            return False
+    sources = [k for k in P if not any(p in P for p in g.producers[k])]
+    src_reads = {img for s in sources for img in g.inputs[s]}
+    for k in P:
+        if k in sources:
+            continue
+        for img in g.inputs[k]:
+            inside = img >= g.n_inputs and (img - g.n_inputs) in P
+            if not inside and img not in src_reads:
+                return False
+    return True
+
+
+def f_mshared(g: Graph, k: int, m: Model) -> float:
+    """Reading O1-h: staged-tile bytes of a local kernel, 0 for a point kernel."""
+    if g.kind[k] != "local":
+        return 0.0
+    return float((m.tile_w + 2 * g.rx[k]) * (m.tile_h + 2 * g.ry[k]) * g.bpp)
+
+
+def _resource_legal(g: Graph, P: set, m: Model) -> bool:
+    """Eq. 2 with fMshared(vP) = sum over the block's local kernels."""
+    loc = [k for k in sorted(P) if g.kind[k] == "local"]
+    if not loc:
+        return True
+    s = 0.0
+    for k in loc:
+        s += f_mshared(g, k, m)
+    mx = max(f_mshared(g, k, m) for k in loc)
+    return s / mx <= m.c_mshared
+
+
+def _header_legal(g: Graph, P: set) -> bool:
+    """Same iteration space is enforced at pipeline creation;
+    access-granularity reading (R-8): the local kernels of one fused block
+    either all use REPEAT or none does."""
+    loc = [k for k in P if g.kind[k] == "local"]
+    rep = [g.mode[k] == "repeat" for k in loc]
+    return all(rep) or not any(rep)
+
+
+def context_legal(g: Graph, P: set, m: Model) -> bool:
+    return _dependence_legal(g, P) and _resource_legal(g, P, m) and _header_legal(g, P)
+
+
+# --------------------------------------------------------------- weights
+
+
+@dataclass
+class EdgeInfo:
+    ks: int
+    kd: int
+    scenario: str     # "point", "p2l", "l2l"
+    w: float          # benefit w + gamma (before clamping)
+    ctx_legal: bool
+    profitable: bool
+    weight: tuple     # (q, eps)
+
+
+def benefit(g: Graph, ks: int, kd: int, m: Model) -> tuple[str, float]:
+    """w for edge (ks, kd) by scenario, Eqs. 3-11, plus gamma (Eq. 12)."""
+    IS = 1.0                                     # reading O1-c
+    n_alu, n_sfu = g.cost[ks]
+    costop = m.c_alu * n_alu + m.c_sfu * n_sfu   # Eq. 6
+    is_ks = float(len(g.inputs[ks]))             # IS_ks: number of input images of ks
+    if g.kind[kd] == "point":                    # point-based, Eq. 5 with Eq. 4
+        return "point", IS * m.tg + m.gamma
+    if m.phi_mode == 1:                          # STAGED reading (O1-g)
+        fac = float((m.tile_w + 2 * g.rx[kd]) * (m.tile_h + 2 * g.ry[kd])) / float(m.tile_w * m.tile_h)
+    elif g.kind[ks] == "point":
+        fac = float((2 * g.rx[kd] + 1) * (2 * g.ry[kd] + 1))           # sz(kd), Eq. 7
+    else:
+        fac = float((2 * g.rx[kd] + 1 + 2 * g.rx[ks]) * (2 * g.ry[kd] + 1 + 2 * g.ry[ks]))  # Eq. 9 (O1-e)
+    phi = costop * is_ks * fac                   # Eq. 7 / Eq. 10
+    if g.kind[ks] == "point":
+        return "p2l", IS * m.tg - phi + m.gamma  # Eq. 8
+    delta_sh = IS * m.tg / m.ts if m.eq3_mode == 0 else IS * (m.tg - m.ts)   # Eq. 3 (O1-a)
+    return "l2l", delta_sh - phi + m.gamma       # Eq. 11
+
+
+def quantize(w: float) -> int:
+    return int(math.floor(w * FIX + 0.5))
+
+
+def edge_weights(g: Graph, m: Model) -> dict:
+    """Alg. 1 lines 2-4: w_e = max(w + gamma, eps) (Eq. 12); illegal -> eps."""
+    info = {}
+    for ks, kd in g.edges:
+        sc, w = benefit(g, ks, kd, m)
+        prof = w > 0.0
+        leg = context_legal(g, {ks, kd}, m)
+        wt = (quantize(w), 0) if (prof and leg) else (0, 1)
+        info[(ks, kd)] = EdgeInfo(ks, kd, sc, w, leg, prof, wt)
+    return info
+
+
+def is_legal(g: Graph, P: set, m: Model, info: dict) -> bool:
+    """IsLegal(p) of Alg. 1 line 9; an unprofitable edge inside forbids the block (O1-g)."""
+    if len(P) == 1:
+        return True
+    for (ks, kd), e in info.items():
+        if ks in P and kd in P and not e.profitable:
+            return False
+    return context_legal(g, P, m)
+
+
+# ---------------------------------------------------------- Stoer-Wagner
+
+
+def _add(a, b):
+    return (a[0] + b[0], a[1] + b[1])
+
+
+def stoer_wagner(g: Graph, P: list, info: dict) -> tuple[list, list, tuple, int]:
+    """Global minimum cut of the undirected view of block P (reading O1-j).
+    Returns (t-side, rest, cut weight, number of phases)."""
+    verts = sorted(P)
+    idx = {v: i for i, v in enumerate(verts)}
+    n = len(verts)
+    W = [[(0, 0)] * n for _ in range(n)]
+    for (ks, kd), e in info.items():
+        if ks in idx and kd in idx:
+            a, b = idx[ks], idx[kd]
+            W[a][b] = _add(W[a][b], e.weight)
+            W[b][a] = _add(W[b][a], e.weight)
+    groups = [[v] for v in verts]
+    active = list(range(n))          # positions in declaration order; merged vertex keeps s's slot
+    best, best_group, phases = None, None, 0
+    while len(active) > 1:
+        phases += 1
+        A = [active[0]]              # start vertex: first active vertex (dx in Fig. 3)
+        conn = {v: W[active[0]][v] for v in active[1:]}
+        last_conn = None
+        while conn:
+            # most tightly connected; ties -> lowest position (first encountered)
+            v = min(conn, key=lambda u: (-conn[u][0], -conn[u][1], active.index(u)))
+            last_conn = conn.pop(v)
+            A.append(v)
+            for u in conn:
+                conn[u] = _add(conn[u], W[v][u])
+        s, t = A[-2], A[-1]
+        if best is None or last_conn < best:      # strict: keep the first one encountered
+            best, best_group = last_conn, list(groups[t])
+        # merge t into s
+        groups[s] = groups[s] + groups[t]
+        for u in range(n):
+            W[s][u] = _add(W[s][u], W[t][u])
+            W[u][s] = _add(W[u][s], W[u][t])
+        W[s][s] = (0, 0)
+        active.remove(t)
+    side = sorted(best_group)
+    rest = sorted(set(verts) - set(side))
+    return side, rest, best, phases
+
+
+# ---------------------------------------------------------------- Alg. 1
+
+
+@dataclass
+class Plan:
+    blocks: list          # lists of kernel ids, topological (by sink)
+    beta: tuple           # (q, eps)
+    info: dict
+    cuts: list            # [(block, side, cut weight, phases)] in processing order
+
+
+def block_weight(P, info) -> tuple:
+    s = (0, 0)
+    for (ks, kd), e in info.items():
+        if ks in P and kd in P:
+            s = _add(s, e.weight)
+    return s
+
+
+def get_legal_partitions(spec: dict, m: Model = PAPER_PROFILE) -> Plan:
+    """Alg. 1 GetLegalPartitions(G)."""
+    g = graph(spec)
+    info = edge_weights(g, m)                  # lines 2-4
+    Sr = []                                    # line 5
+    Sp = [list(range(g.n))]                    # line 6
+    cuts = []
+    while Sp:                                  # lines 7-17
+        p = Sp.pop(0)
+        if len(p) == 1 or is_legal(g, set(p), m, info):
+            Sr.append(p)
+        else:
+            a, b, w, ph = stoer_wagner(g, p, info)
+            cuts.append((p, a, w, ph))
+            Sp += [a, b]
+    Sr.sort(key=max)
+    beta = (0, 0)
+    for P in Sr:
+        beta = _add(beta, block_weight(set(P), info))
+    return Plan(Sr, beta, info, cuts)
+
+
+# ------------------------------------------------------------ brute force
+
+
+def _connected(g: Graph, P: list) -> bool:
+    S = set(P)
+    seen, stack = {P[0]}, [P[0]]
+    while stack:
+        v = stack.pop()
+        for u in g.consumers[v] + g.producers[v]:
+            if u in S and u not in seen:
+                seen.add(u)
+                stack.append(u)
+    return len(seen) == len(S)
+
+
+def brute_force(spec: dict, m: Model = PAPER_PROFILE) -> tuple[tuple, list]:
+    """Maximum of Eq. 1 over all partitions into connected legal blocks
+    (restricted-growth enumeration; Bell(n) partitions)."""
+    g = graph(spec)
+    info = edge_weights(g, m)
+    n = g.n
+    memo = {}
+
+    def ok(block):
+        key = frozenset(block)
+        if key not in memo:
+            memo[key] = (len(block) == 1 or (_connected(g, block) and is_legal(g, key, m, info)))
+        return memo[key]
+
+    best = [None, None]
+    blocks: list[list[int]] = []
+
+    # enumerate and check legality on completion
+    def rec2(i):
+        if i == n:
+            if all(ok(b) for b in blocks):
+                val = (0, 0)
+                for b in blocks:
+                    val = _add(val, block_weight(set(b), info))
+                if best[0] is None or val > best[0]:
+                    best[0], best[1] = val, sorted([sorted(b) for b in blocks], key=max)
+            return
+        for b in blocks:
+            b.append(i)
+            rec2(i + 1)
+            b.pop()
+        blocks.append([i])
+        rec2(i + 1)
+        blocks.pop()
+
+    rec2(0)
+    return best[0], best[1]
+
+
+def min_cut_brute(g: Graph, P: list, info: dict) -> tuple:
+    """Textbook check for Stoer-Wagner: min over all 2^(n-1)-1 bipartitions."""
+    verts = sorted(P)
+    n = len(verts)
+    best = None
+    for mask in range(1, 1 << (n - 1)):
+        S = {verts[i] for i in range(n) if mask >> i & 1}
+        w = (0, 0)
+        for (ks, kd), e in info.items():
+            if ks in P and kd in P and ((ks in S) != (kd in S)):
+                w = _add(w, e.weight)
+        if best is None or w < best:
+            best = w
+    return best
