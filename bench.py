@@ -1,0 +1,367 @@
+#!/usr/bin/env python
+"""Benchmark of the fused image-pipeline hot path on B200 (BASELINE.json metric:
+"Harris 4096^2 Mpixel/s fused vs unfused; DRAM bytes/pixel; HBM GB/s vs peak").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl kfuse|reference]
+                    [--config C3] [--plan b200]
+
+N=1: workload C3 = Harris 4096x4096 float32 (clamp), the B200-profile plan
+(fully fused, one launch per step).  A step = one kf_run over one image, inputs
+already resident in HBM; 4 rotating input/output buffer sets (512 MiB > the
+126 MB L2) so consecutive steps never hit in L2.  The unfused (9 launches) and
+paper-profile (6 launches) plans are timed the same way and reported beside it.
+N>1 (torchrun): weak scaling by row bands, each rank a 4096x4096 band of a
+(4096N)x4096 image; every step = one NCCL halo-row exchange + kf_run_band.
+--impl reference: the unfused CPU oracle (oracle/) timed on the host cores.
+One JSON line on stdout (rank 0).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "Harris 4096² Mpixel/s fused vs unfused; DRAM bytes/pixel; HBM GB/s vs peak"
+UNIT = "Mpixel/s"
+DATA = "synthetic: counter-based SplitMix64 uniform [0,1) images (kf_inputs/gen.py), as the paper's random images"
+# algorithmic DRAM bytes per pixel of each plan: every launched kernel
+# reads its external inputs once and writes its output once (f32: 4 B per image)
+ALG_BYTES = {"harris": {"unfused": 84, "paper": 60, "b200": 8},
+             "shitomasi": {"unfused": 84, "paper": 60, "b200": 8},
+             "unsharp": {"unfused": 44, "paper": 8, "b200": 8},
+             "deep10": {"unfused": 100, "paper": 92, "b200": 8}}
+
+
+def load_peaks() -> dict:
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+    except Exception:
+        return {"hbm_gbs": 6650.0, "source": "fallback 6.65 TB/s (B200_PROFILING.md)"}
+
+
+def ncu_traffic(cfg: str, plan: str):
+    """dram bytes per launch from the committed ncu --set full summary, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(path) as f:
+            d = json.load(f)
+        return d.get(f"{cfg}:{plan}")
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """NVML samples of SM clock and throttle reasons during the timed region."""
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception:
+            self.nv = None
+
+    def _sample(self):
+        nv = self.nv
+        self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+        r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        for bit, name in self.REASONS.items():
+            if r & bit and name != "gpu_idle":
+                self.reasons.add(name)
+
+    def _loop(self):
+        while not self._stop.is_set():
+            try:
+                self._sample()
+            except Exception:
+                return
+            time.sleep(0.002)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._loop, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        if self.nv:
+            self._stop.set()
+            self.t.join()
+            if not self.samples:
+                self._sample()
+
+    def summary(self) -> dict:
+        if not self.nv:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ----------------------------------------------------------------- reference
+
+
+def cpu_oracle_run(workload: str, width: int, rows: int, seed: int) -> tuple[float, int]:
+    """Times the unfused oracle on a width x rows image; returns (seconds, pixels)."""
+    from kf_inputs import gen
+    from kf_inputs import pipelines as P
+    from oracle import oracle as O
+    spec = P.WORKLOADS[workload](width, rows)
+    ins = [gen.image(spec["dtype"], seed, width, rows)]
+    t = time.perf_counter()
+    O.run(spec, ins)
+    return time.perf_counter() - t, width * rows
+
+
+def run_reference(args, cfg_name, spec) -> None:
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    rows = 128 if spec["dtype"] == "f32" else 32
+    for _ in range(args.warmup):
+        cpu_oracle_run(spec["name"], spec["width"], rows, 1)
+    tot, px = 0.0, 0
+    for _ in range(args.steps):
+        dt, n = cpu_oracle_run(spec["name"], spec["width"], rows, 1)
+        tot += dt
+        px += n
+    v = px / tot / 1e6
+    sample = f"{spec['width']}x{rows} strip of the {spec['width']}x{spec['height']} {spec['name']} workload per step"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot / args.steps * 1e3, 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": DATA, "config": config_dict(cfg_name, spec, "unfused-oracle"),
+        "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }))
+
+
+def config_dict(cfg_name, spec, plan, extra=None) -> dict:
+    d = {"workload": f"{cfg_name}: {spec['name']} {spec['width']}x{spec['height']} {spec['dtype']}",
+         "width": spec["width"], "height": spec["height"], "plan": plan,
+         "l2": "4 rotating input/output buffer sets (512 MiB) > 126 MB L2"}
+    if extra:
+        d.update(extra)
+    return d
+
+
+# --------------------------------------------------------------------- GPU
+
+
+def time_plan(plan, ins, outs, steps, warmup, stream, torch, launches):
+    """Times exactly `steps` kf_run calls; returns (ms/step total, mean per-step
+    event time of the plan's kernels)."""
+    n = len(ins)
+    with torch.cuda.stream(stream):
+        for i in range(warmup):
+            plan.run([ins[i % n]], [outs[i % n]], stream)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t0.record(stream)
+    for i in range(steps):
+        ev[i][0].record(stream)
+        plan.run([ins[i % n]], [outs[i % n]], stream)
+        ev[i][1].record(stream)
+    t1.record(stream)
+    torch.cuda.synchronize()
+    per = [a.elapsed_time(b) for a, b in ev]
+    return t0.elapsed_time(t1) / steps, sum(per) / len(per)
+
+
+def bench_single(args, cfg_name, spec, seed) -> None:
+    import torch
+
+    from kf_inputs import gen
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+
+    dev = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(dev)
+    W, H = spec["width"], spec["height"]
+    px = W * H
+    host = gen.image(spec["dtype"], seed, W, H)
+    tdt = torch.float32 if spec["dtype"] == "f32" else torch.uint8
+    oshape = (H, W) if spec["dtype"] == "f32" else (H, W, 4)
+    nsets = 4
+    ins = [torch.from_numpy(host).cuda() for _ in range(nsets)]
+    outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(nsets)]
+    stream = torch.cuda.Stream()
+    results = {}
+    plans = {}
+    for kind in ("unfused", "paper", "b200"):
+        p = K.Pipeline.from_spec(spec)
+        plan = p.plan_unfused() if kind == "unfused" else p.plan_fusion(kind)
+        plan.prepare()
+        plans[kind] = (p, plan)
+    # headline plan last, with clocks sampled during its timed region
+    order = [k for k in ("unfused", "paper", "b200") if k != args.plan] + [args.plan]
+    clocks = None
+    for kind in order:
+        p, plan = plans[kind]
+        if kind == args.plan:
+            with ClockSampler(dev) as cs:
+                ms, kern_ms = time_plan(plan, ins, outs, args.steps, args.warmup, stream, torch, plan.num_launches)
+            clocks = cs.summary()
+        else:
+            ms, kern_ms = time_plan(plan, ins, outs, max(20, args.steps // 4), args.warmup, stream, torch,
+                                    plan.num_launches)
+        ab = ALG_BYTES.get(spec["name"], {}).get(kind)
+        results[kind] = {"ms_per_step": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
+                         "launches": plan.num_launches, "alg_bytes_per_px": ab,
+                         "alg_gbs": round(ab * px / (ms * 1e-3) / 1e9, 1) if ab else None,
+                         "kernel_ms": round(kern_ms, 5)}
+    head = results[args.plan]
+    peaks = load_peaks()
+    _, hplan = plans[args.plan]
+    ab = head["alg_bytes_per_px"] or 8
+    achieved = ab * px / (head["kernel_ms"] * 1e-3) / 1e9
+    traffic = ncu_traffic(cfg_name, args.plan)
+    roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
+                "peak_source": peaks["source"],
+                "per_launch": f"{ab} B/px x {px} px = {ab * px} algorithmic bytes per launch"}
+    # end to end through the public API with host buffers (pinned)
+    e2e_steps = max(3, min(args.steps, 20))
+    hin = torch.from_numpy(host).pin_memory()
+    hout = torch.empty(oshape, dtype=tdt).pin_memory()
+    for _ in range(2):
+        hplan.run_host([hin], [hout], stream)
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    for _ in range(e2e_steps):
+        hplan.run_host([hin], [hout], stream)
+    e2e_s = (time.perf_counter() - t) / e2e_steps
+    e2e = {"value": round(px / e2e_s / 1e6, 1), "unit": UNIT, "h2d_bytes_per_step": int(hin.numel() * hin.element_size()),
+           "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps}
+    # CPU baseline: the unfused oracle on this box's host, one full image
+    cpu = None
+    if not args.no_cpu:
+        dt, n = cpu_oracle_run(spec["name"], W, H if spec["dtype"] == "f32" else 256, seed)
+        cpu = {"value": round(n / dt / 1e6, 3), "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": f"one {W}x{H if spec['dtype'] == 'f32' else 256} image of the workload, unfused fp64 oracle, 1 thread"}
+    out = {
+        "metric": METRIC, "value": head["mpix_s"], "unit": UNIT, "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": head["ms_per_step"], "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32" if spec["dtype"] == "f32" else "u8x4/int32", "data": DATA,
+        "config": config_dict(cfg_name, spec, args.plan),
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+        "gpu_launches": args.steps * hplan.num_launches, "clocks": clocks,
+        "plans": results,
+        "fused_vs_unfused": round(results["unfused"]["ms_per_step"] / head["ms_per_step"], 3),
+    }
+    print(json.dumps(out))
+
+
+def bench_multi(args, cfg_name, spec, seed) -> None:
+    import torch
+    import torch.distributed as dist
+
+    from kf_inputs import gen
+    from kf_inputs import pipelines as P
+    from paper_conf_cgo_qiaorht19_b200 import dist as KD
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+
+    dist.init_process_group("nccl")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    dev = int(os.environ.get("LOCAL_RANK", rank))
+    torch.cuda.set_device(dev)
+    W, Hb = spec["width"], spec["height"]
+    Htot = Hb * world                                 # weak scaling: one band per GPU
+    gspec = P.WORKLOADS[spec["name"]](W, Htot)
+    p = K.Pipeline.from_spec(gspec)
+    plan = p.plan_unfused() if args.plan == "unfused" else p.plan_fusion(args.plan)
+    plan.prepare()
+    band = KD.partition(Htot, world, rank, plan.halo_rows)
+    host = gen.image(gspec["dtype"], seed, W, Htot, band.in0, band.in1)
+    tdt = torch.float32 if gspec["dtype"] == "f32" else torch.uint8
+    nsets = 4
+    ins = [torch.from_numpy(host).cuda() for _ in range(nsets)]
+    oshape = (band.rows, W) if gspec["dtype"] == "f32" else (band.rows, W, 4)
+    outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(nsets)]
+    stream = torch.cuda.current_stream()
+
+    def step(i):
+        KD.exchange_halos(ins[i % nsets], band)
+        KD.run_band(plan, band, [ins[i % nsets]], [outs[i % nsets]], stream)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    dist.barrier()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(dev) as cs:
+        t0.record()
+        for i in range(args.steps):
+            step(i)
+        t1.record()
+        torch.cuda.synchronize()
+    dist.barrier()
+    ms = torch.tensor([t0.elapsed_time(t1) / args.steps], device="cuda")
+    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+    ms = float(ms.item())
+    px = W * Htot
+    if rank == 0:
+        ab = ALG_BYTES.get(gspec["name"], {}).get(args.plan) or 8
+        peaks = load_peaks()
+        ach = ab * (band.rows * W) / (ms * 1e-3) / 1e9
+        print(json.dumps({
+            "metric": METRIC, "value": round(px / (ms * 1e-3) / 1e6, 1), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": DATA,
+            "config": config_dict(cfg_name, gspec, args.plan,
+                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows via NCCL send/recv",
+                                   "band": f"{Hb}x{W} per GPU"}),
+            "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                         "frac": round(ach / peaks["hbm_gbs"], 4), "traffic": None,
+                         "peak_source": peaks["source"], "note": "per GPU, step time incl. halo exchange"},
+            "cpu_baseline": None,
+            "e2e": None,
+            "gpu_launches": args.steps * plan.num_launches, "clocks": cs.summary(),
+        }))
+    dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="kfuse", choices=["kfuse", "reference"])
+    ap.add_argument("--config", default="C3")
+    ap.add_argument("--plan", default="b200", choices=["b200", "paper", "unfused"])
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    from kf_inputs import pipelines as P
+    spec, seed = P.config(args.config)
+    if args.impl == "reference":
+        run_reference(args, args.config, spec)
+        return
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1:
+        bench_multi(args, args.config, spec, seed)
+    else:
+        bench_single(args, args.config, spec, seed)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,148 @@
+// kf_device.cuh -- device-side library included by every generated fused
+// kernel (compiled by NVRTC for sm_100a).  Hand-written; the code generator
+// (codegen.cpp) only emits the per-block glue that calls into it.
+//
+// Value types: KF_F32 pipelines compute in float; KF_U8X4 pipelines compute per
+// channel in int32 (struct I4) and store saturated uchar4 (PAPER.md:1051-1053:
+// the intermediate becomes a register; narrowing at every kernel
+// boundary, kept in the fused kernel).
+#pragma once
+
+#define KF_MAX_IMG 16
+
+struct KfArgs {
+    const void *img[KF_MAX_IMG];   // external images of the block (slot order)
+    int base[KF_MAX_IMG];          // global row held by row 0 of each buffer
+    void *out;                     // block output image
+    int out_base;                  // global row held by row 0 of `out`
+    int W, H;                      // image size (global)
+    int r0, r1;                    // output rows computed by this launch
+    int tiles_x;                   // v1 tiling
+    int tiles_y;
+};
+
+// ------------------------------------------------------------ border map
+// Per-axis index map of PAPER.md:1050-1052 (clamp / mirror / repeat) plus
+// mirror101 and constant, folded until in range.  -1 = use the constant.
+enum { KF_B_CLAMP = 0, KF_B_MIRROR = 1, KF_B_MIRROR101 = 2, KF_B_REPEAT = 3, KF_B_CONSTANT = 4 };
+
+template <int MODE>
+__device__ __forceinline__ int kf_border(int p, int n)
+{
+    if (MODE == KF_B_CLAMP) return min(max(p, 0), n - 1);
+    if (MODE == KF_B_CONSTANT) return (p >= 0 && p < n) ? p : -1;
+    if (MODE == KF_B_REPEAT) { int r = p % n; return r < 0 ? r + n : r; }
+    if (MODE == KF_B_MIRROR) {
+        while (p < 0 || p >= n) p = (p < 0) ? -p - 1 : 2 * n - p - 1;
+        return p;
+    }
+    // MIRROR101
+    if (n == 1) return 0;
+    while (p < 0 || p >= n) p = (p < 0) ? -p : 2 * n - p - 2;
+    return p;
+}
+
+__device__ __forceinline__ int kf_wrap(int p, int n) { int r = p % n; return r < 0 ? r + n : r; }
+
+// ------------------------------------------------------------- I4 (u8x4)
+struct I4 { int x, y, z, w; };
+
+__device__ __forceinline__ I4 kf_i4(int v) { return I4{v, v, v, v}; }
+__device__ __forceinline__ I4 kf_unpack(unsigned u)
+{
+    return I4{(int)(u & 0xffu), (int)((u >> 8) & 0xffu), (int)((u >> 16) & 0xffu), (int)(u >> 24)};
+}
+__device__ __forceinline__ int kf_sat(int v) { return min(max(v, 0), 255); }
+__device__ __forceinline__ unsigned kf_pack(I4 a)
+{
+    return (unsigned)kf_sat(a.x) | ((unsigned)kf_sat(a.y) << 8) | ((unsigned)kf_sat(a.z) << 16) |
+           ((unsigned)kf_sat(a.w) << 24);
+}
+
+#define KF_I4_BIN(name, expr)                                                              \
+    __device__ __forceinline__ I4 name(I4 a, I4 b)                                         \
+    {                                                                                      \
+        I4 r;                                                                              \
+        { int A = a.x, B = b.x; r.x = (expr); }                                            \
+        { int A = a.y, B = b.y; r.y = (expr); }                                            \
+        { int A = a.z, B = b.z; r.z = (expr); }                                            \
+        { int A = a.w, B = b.w; r.w = (expr); }                                            \
+        return r;                                                                          \
+    }
+#define KF_I4_UN(name, expr)                                                               \
+    __device__ __forceinline__ I4 name(I4 a)                                               \
+    {                                                                                      \
+        I4 r;                                                                              \
+        { int A = a.x; r.x = (expr); }                                                     \
+        { int A = a.y; r.y = (expr); }                                                     \
+        { int A = a.z; r.z = (expr); }                                                     \
+        { int A = a.w; r.w = (expr); }                                                     \
+        return r;                                                                          \
+    }
+
+KF_I4_BIN(kf_add, A + B)
+KF_I4_BIN(kf_sub, A - B)
+KF_I4_BIN(kf_mul, A * B)
+KF_I4_BIN(kf_div, B == 0 ? 0 : A / B)
+KF_I4_BIN(kf_min, min(A, B))
+KF_I4_BIN(kf_max, max(A, B))
+KF_I4_UN(kf_abs, abs(A))
+KF_I4_UN(kf_neg, -A)
+KF_I4_UN(kf_satu8, kf_sat(A))
+
+template <int N> __device__ __forceinline__ I4 kf_shr(I4 a) { return I4{a.x >> N, a.y >> N, a.z >> N, a.w >> N}; }
+template <int N> __device__ __forceinline__ I4 kf_shl(I4 a)
+{
+    return I4{(int)((unsigned)a.x << N), (int)((unsigned)a.y << N), (int)((unsigned)a.z << N),
+              (int)((unsigned)a.w << N)};
+}
+__device__ __forceinline__ I4 kf_clamp(I4 a, I4 lo, I4 hi) { return kf_min(kf_max(a, lo), hi); }
+__device__ __forceinline__ I4 kf_sel_gt(I4 a, I4 b, I4 c, I4 d)
+{
+    return I4{a.x > b.x ? c.x : d.x, a.y > b.y ? c.y : d.y, a.z > b.z ? c.z : d.z, a.w > b.w ? c.w : d.w};
+}
+__device__ __forceinline__ I4 kf_lut(I4 a, const int *__restrict__ t, int n)
+{
+    return I4{__ldg(t + min(max(a.x, 0), n - 1)), __ldg(t + min(max(a.y, 0), n - 1)),
+              __ldg(t + min(max(a.z, 0), n - 1)), __ldg(t + min(max(a.w, 0), n - 1))};
+}
+// multiply-accumulate with an integer mask coefficient
+__device__ __forceinline__ I4 kf_mac(I4 acc, int m, I4 v)
+{
+    return I4{acc.x + m * v.x, acc.y + m * v.y, acc.z + m * v.z, acc.w + m * v.w};
+}
+
+// -------------------------------------------------------------- float
+__device__ __forceinline__ float kf_add(float a, float b) { return a + b; }
+__device__ __forceinline__ float kf_sub(float a, float b) { return a - b; }
+__device__ __forceinline__ float kf_mul(float a, float b) { return a * b; }
+__device__ __forceinline__ float kf_div(float a, float b) { return a / b; }
+__device__ __forceinline__ float kf_min(float a, float b) { return fminf(a, b); }
+__device__ __forceinline__ float kf_max(float a, float b) { return fmaxf(a, b); }
+__device__ __forceinline__ float kf_abs(float a) { return fabsf(a); }
+__device__ __forceinline__ float kf_neg(float a) { return -a; }
+__device__ __forceinline__ float kf_sqrt(float a) { return sqrtf(a); }
+__device__ __forceinline__ float kf_exp(float a) { return expf(a); }
+__device__ __forceinline__ float kf_log(float a) { return logf(a); }
+__device__ __forceinline__ float kf_pow(float a, float b) { return powf(a, b); }
+__device__ __forceinline__ float kf_clamp(float a, float lo, float hi) { return fminf(fmaxf(a, lo), hi); }
+__device__ __forceinline__ float kf_sel_gt(float a, float b, float c, float d) { return a > b ? c : d; }
+__device__ __forceinline__ float kf_mac(float acc, float m, float v) { return fmaf(m, v, acc); }
+
+// ------------------------------------------------------ global image access
+__device__ __forceinline__ float kf_ldf(const void *p, int base, int W, int y, int x)
+{
+    return __ldg((const float *)p + (size_t)(y - base) * W + x);
+}
+__device__ __forceinline__ I4 kf_ldi(const void *p, int base, int W, int y, int x)
+{
+    return kf_unpack(__ldg((const unsigned *)p + (size_t)(y - base) * W + x));
+}
+__device__ __forceinline__ void kf_stf(void *p, int base, int W, int y, int x, float v)
+{
+    ((float *)p)[(size_t)(y - base) * W + x] = v;
+}
+__device__ __forceinline__ void kf_sti(void *p, int base, int W, int y, int x, I4 v)
+{
+    ((unsigned *)p)[(size_t)(y - base) * W + x] = kf_pack(v);
+}

@@ -1,0 +1,135 @@
+// kf_internal.h -- host-side data structures of libkfuse (not part of the ABI).
+#pragma once
+
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "../../include/kfuse.h"
+
+namespace kf {
+
+// ---- error plumbing: a thrown kf::Error becomes a kf_status at the C boundary
+struct Error {
+    kf_status st;
+    std::string msg;
+};
+[[noreturn]] void fail(kf_status st, const std::string &msg);
+void set_error(const std::string &msg);
+
+struct Instr {
+    int op, arg;
+    double imm;
+};
+
+enum Kind { POINT = 0, LOCAL = 1 };
+
+struct Op {
+    Kind kind = POINT;
+    std::vector<int> inputs;      // image ids; LOCAL: exactly one
+    std::vector<Instr> prog;      // POINT: body; LOCAL: post program on ACC (empty = identity)
+    std::vector<int> lut;
+    int mw = 0, mh = 0;           // LOCAL mask size (odd)
+    std::vector<double> mask;     // row-major mh x mw
+    int mode = KF_CLAMP;
+    double constant = 0.0;
+    int n_alu = 0, n_sfu = 0;     // Eq. 6 costs
+    int rx() const { return kind == LOCAL ? mw / 2 : 0; }
+    int ry() const { return kind == LOCAL ? mh / 2 : 0; }
+};
+
+struct Runtime;   // runtime.cu
+
+}  // namespace kf
+
+struct kf_pipeline {
+    int W = 0, H = 0, dtype = KF_F32;
+    int n_inputs = 0;
+    std::vector<kf::Op> ops;
+    std::vector<int> outputs;     // marked output image ids, in marking order
+    bool frozen = false;
+    kf::Runtime *rt = nullptr;    // owned; created lazily by the runtime
+    ~kf_pipeline();
+    int n_images() const { return n_inputs + (int)ops.size(); }
+    bool is_kernel_image(int id) const { return id >= n_inputs; }
+};
+
+namespace kf {
+
+struct EdgeInfo {
+    int ks, kd;
+    int scenario;                 // 0 point-based, 1 point-to-local, 2 local-to-local
+    double w;                     // benefit incl. gamma, before clamping (Eq. 12)
+    bool ctx_legal, profitable;
+    int64_t q, eps;               // weight as lexicographic pair
+};
+
+struct CutInfo {
+    std::vector<int> side;
+    int64_t q, eps;
+    int phases;
+};
+
+// Block analysis shared by code generation and the executor.
+struct BlockInfo {
+    std::vector<int> kernels;     // ascending kernel ids
+    int sink = -1;                // kernel id
+    std::vector<int> ext;         // external images read (ascending image ids)
+    std::map<int, int> hx, hy;    // halo of each kernel's OUTPUT needed inside the block
+    std::map<int, int> ext_hx, ext_hy;  // halo of each external image
+    std::set<int> staged;         // kernels consumed by an in-block local kernel
+    bool torus = false;           // all local kernels REPEAT: slot model
+    int Rx = 0, Ry = 0;           // max external halo
+};
+
+struct CompiledBlock;             // runtime.cu
+
+}  // namespace kf
+
+struct kf_plan {
+    kf_pipeline *pipe = nullptr;
+    std::vector<std::vector<int>> blocks;    // topological (by sink)
+    int64_t beta_q = 0, beta_eps = 0;
+    std::vector<kf::EdgeInfo> edges;
+    std::vector<kf::CutInfo> cuts;
+    std::vector<kf::BlockInfo> info;         // per block
+    int halo_rows = 0;
+    // runtime state (runtime.cu)
+    std::vector<std::shared_ptr<kf::CompiledBlock>> compiled;
+    std::map<int, void *> workspace;         // image id -> device buffer (cut edges)
+    bool prepared = false;
+    ~kf_plan();
+};
+
+namespace kf {
+
+// graph.cpp
+void validate_program(const kf_pipeline *p, const std::vector<Instr> &prog, int n_loads, bool has_lut);
+void default_cost(const kf_pipeline *p, Op &op);
+std::vector<std::vector<int>> consumers(const kf_pipeline *p);   // kernel -> consumer kernels
+std::vector<std::vector<int>> producers(const kf_pipeline *p);   // kernel -> producer kernels
+
+// planner.cpp
+kf_plan *plan_fusion(kf_pipeline *p, const kf_model_params &m);
+kf_plan *plan_from_blocks(kf_pipeline *p, std::vector<std::vector<int>> blocks, bool check);
+bool dependence_legal(const kf_pipeline *p, const std::set<int> &P);
+bool header_legal(const kf_pipeline *p, const std::set<int> &P);
+BlockInfo analyse_block(const kf_pipeline *p, const std::vector<int> &kernels);
+
+// codegen.cpp
+std::string kernel_name(int block);
+std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block, int tile_w, int tile_h);
+
+// runtime.cu
+void prepare(kf_pipeline *p, kf_plan *plan);
+void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
+         void *stream, int row0, int row1, int in_row0);
+void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
+              void *stream);
+void release_plan(kf_plan *plan);
+void release_runtime(kf_pipeline *p);
+
+}  // namespace kf

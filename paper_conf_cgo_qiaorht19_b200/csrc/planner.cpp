@@ -1,0 +1,361 @@
+// planner.cpp -- the fusion planner of Qiao et al. (CGO'19), host side.
+//
+//   edge weights   Eqs. 3-12, scenario per edge
+//   IsLegal        dependence (Fig. 2), resources (Eq. 2,
+//                  PAPER.md:296-321), header, profitability
+//
+//   MinCut         Stoer-Wagner [14] on the undirected view
+//   Alg. 1         GetLegalPartitions
+//
+// Readings of the garbled/silent passages are listed in DESIGN.md §3 (R-1..R-9).
+// Weights are lexicographic pairs (q, eps): q = floor(w * 2^20 + 0.5) in
+// fixed point so that sums and ties are exact (R-9), eps counts the
+// "arbitrarily small positive" weights of illegal edges.
+#include <algorithm>
+#include <cmath>
+#include <deque>
+#include <functional>
+
+#include "kf_internal.h"
+
+namespace kf {
+
+namespace {
+
+struct W2 {
+    int64_t q = 0, e = 0;
+    W2 operator+(const W2 &o) const { return {q + o.q, e + o.e}; }
+    bool operator<(const W2 &o) const { return q != o.q ? q < o.q : e < o.e; }
+};
+
+int64_t quantize(double w) { return (int64_t)std::floor(w * 1048576.0 + 0.5); }
+
+double f_mshared(const kf_pipeline *p, int k, const kf_model_params &m)
+{
+    const Op &o = p->ops[k];
+    if (o.kind != LOCAL) return 0.0;
+    return (double)((int64_t)(m.tile_w + 2 * o.rx()) * (m.tile_h + 2 * o.ry()) * 4);
+}
+
+}  // namespace
+
+// Fig. 2 reading (R-1): exactly one sink kd; every other kernel has
+// all its consumers inside and is not a pipeline output (2c); every image a
+// non-source kernel reads from outside is also read by a source kernel (2b vs 2d).
+bool dependence_legal(const kf_pipeline *p, const std::set<int> &P)
+{
+    auto co = consumers(p);
+    auto pr = producers(p);
+    int sink = -1, nsink = 0;
+    for (int k : P) {
+        bool inner = false;
+        for (int c : co[k]) inner |= P.count(c) > 0;
+        if (!inner) { sink = k; nsink++; }
+    }
+    if (nsink != 1) return false;
+    std::set<int> outs(p->outputs.begin(), p->outputs.end());
+    for (int k : P) {
+        if (k == sink) continue;
+        if (outs.count(p->n_inputs + k)) return false;
+        for (int c : co[k])
+            if (!P.count(c)) return false;
+    }
+    std::set<int> src_reads;
+    std::set<int> sources;
+    for (int k : P) {
+        bool has_prod = false;
+        for (int s : pr[k]) has_prod |= P.count(s) > 0;
+        if (!has_prod) {
+            sources.insert(k);
+            for (int img : p->ops[k].inputs) src_reads.insert(img);
+        }
+    }
+    for (int k : P) {
+        if (sources.count(k)) continue;
+        for (int img : p->ops[k].inputs) {
+            bool inside = img >= p->n_inputs && P.count(img - p->n_inputs);
+            if (!inside && !src_reads.count(img)) return false;
+        }
+    }
+    return true;
+}
+
+// Eq. 2 with fMshared(vP) = sum of the block's local kernels' staged tiles (R-2).
+static bool resource_legal(const kf_pipeline *p, const std::set<int> &P, const kf_model_params &m)
+{
+    double s = 0.0, mx = 0.0;
+    bool any = false;
+    for (int k : P) {               // std::set iterates ascending, as the reference does
+        if (p->ops[k].kind != LOCAL) continue;
+        any = true;
+        s += f_mshared(p, k, m);
+        mx = std::max(mx, f_mshared(p, k, m));
+    }
+    if (!any) return true;
+    return s / mx <= m.c_mshared;
+}
+
+// Header compatibility: one iteration space per pipeline is
+// enforced at creation; access-granularity reading R-8: the local kernels of a
+// fused block all use REPEAT or none does.
+bool header_legal(const kf_pipeline *p, const std::set<int> &P)
+{
+    int rep = 0, loc = 0;
+    for (int k : P)
+        if (p->ops[k].kind == LOCAL) {
+            loc++;
+            rep += p->ops[k].mode == KF_REPEAT;
+        }
+    return rep == 0 || rep == loc;
+}
+
+static bool context_legal(const kf_pipeline *p, const std::set<int> &P, const kf_model_params &m)
+{
+    return dependence_legal(p, P) && resource_legal(p, P, m) && header_legal(p, P);
+}
+
+// Benefit of one edge, Eqs. 3-11 plus gamma (Eq. 12 before clamping).
+static EdgeInfo benefit(const kf_pipeline *p, int ks, int kd, const kf_model_params &m)
+{
+    const Op &s = p->ops[ks], &d = p->ops[kd];
+    const double IS = 1.0;                                    // R-5
+    const double costop = m.c_alu * s.n_alu + m.c_sfu * s.n_sfu;   // Eq. 6
+    const double is_ks = (double)s.inputs.size();
+    EdgeInfo e{};
+    e.ks = ks;
+    e.kd = kd;
+    if (d.kind == POINT) {                                    // point-based, Eqs. 4-5
+        e.scenario = 0;
+        e.w = IS * m.tg + m.gamma;
+        return e;
+    }
+    double fac;
+    if (m.phi_mode == 1)                                      // STAGED (R-4)
+        fac = (double)((m.tile_w + 2 * d.rx()) * (m.tile_h + 2 * d.ry())) / (double)(m.tile_w * m.tile_h);
+    else if (s.kind == POINT)
+        fac = (double)((2 * d.rx() + 1) * (2 * d.ry() + 1)); // sz(kd), Eq. 7
+    else
+        fac = (double)((2 * d.rx() + 1 + 2 * s.rx()) * (2 * d.ry() + 1 + 2 * s.ry()));  // Eq. 9 (R-6)
+    const double phi = costop * is_ks * fac;                  // Eqs. 7 / 10
+    if (s.kind == POINT) {
+        e.scenario = 1;
+        e.w = IS * m.tg - phi + m.gamma;                      // Eq. 8
+    } else {
+        e.scenario = 2;
+        double dsh = m.eq3_mode == 0 ? IS * m.tg / m.ts : IS * (m.tg - m.ts);   // Eq. 3 (R-7)
+        e.w = dsh - phi + m.gamma;                            // Eq. 11
+    }
+    return e;
+}
+
+static std::vector<EdgeInfo> edge_weights(const kf_pipeline *p, const kf_model_params &m)
+{
+    std::vector<EdgeInfo> out;
+    auto pr = producers(p);
+    for (int kd = 0; kd < (int)p->ops.size(); kd++)
+        for (int ks : pr[kd]) {
+            EdgeInfo e = benefit(p, ks, kd, m);
+            e.profitable = e.w > 0.0;
+            e.ctx_legal = context_legal(p, {ks, kd}, m);
+            if (e.profitable && e.ctx_legal) { e.q = quantize(e.w); e.eps = 0; }
+            else { e.q = 0; e.eps = 1; }                      // w_e = eps (Eq. 12)
+            out.push_back(e);
+        }
+    return out;
+}
+
+static bool is_legal(const kf_pipeline *p, const std::set<int> &P, const kf_model_params &m,
+                     const std::vector<EdgeInfo> &E)
+{
+    if (P.size() == 1) return true;
+    for (const EdgeInfo &e : E)
+        if (P.count(e.ks) && P.count(e.kd) && !e.profitable) return false;   // R-3
+    return context_legal(p, P, m);
+}
+
+// Stoer-Wagner global minimum cut with the deterministic tie-breaks of R-9:
+// start vertex = first active vertex in declaration order, most tightly
+// connected next (ties: lowest declaration index), merged vertex keeps s's
+// slot, keep the first minimum encountered (strict <).
+static CutInfo stoer_wagner(const std::vector<int> &verts, const std::vector<EdgeInfo> &E)
+{
+    const int n = (int)verts.size();
+    std::map<int, int> idx;
+    for (int i = 0; i < n; i++) idx[verts[i]] = i;
+    std::vector<std::vector<W2>> Wm(n, std::vector<W2>(n));
+    for (const EdgeInfo &e : E) {
+        auto a = idx.find(e.ks), b = idx.find(e.kd);
+        if (a == idx.end() || b == idx.end()) continue;
+        W2 w{e.q, e.eps};
+        Wm[a->second][b->second] = Wm[a->second][b->second] + w;
+        Wm[b->second][a->second] = Wm[b->second][a->second] + w;
+    }
+    std::vector<std::vector<int>> groups(n);
+    for (int i = 0; i < n; i++) groups[i] = {verts[i]};
+    std::vector<int> active(n);
+    for (int i = 0; i < n; i++) active[i] = i;
+    bool have = false;
+    W2 best;
+    std::vector<int> best_group;
+    int phases = 0;
+    while (active.size() > 1) {
+        phases++;
+        std::vector<int> A{active[0]};
+        std::vector<int> rest(active.begin() + 1, active.end());   // ascending positions
+        std::vector<W2> conn(n);
+        for (int v : rest) conn[v] = Wm[active[0]][v];
+        W2 last;
+        while (!rest.empty()) {
+            size_t bi = 0;
+            for (size_t i = 1; i < rest.size(); i++)
+                if (conn[rest[bi]] < conn[rest[i]]) bi = i;      // strictly larger wins; ties keep lowest
+            int v = rest[bi];
+            last = conn[v];
+            rest.erase(rest.begin() + bi);
+            A.push_back(v);
+            for (int u : rest) conn[u] = conn[u] + Wm[v][u];
+        }
+        int s = A[A.size() - 2], t = A.back();
+        if (!have || last < best) {
+            have = true;
+            best = last;
+            best_group = groups[t];
+        }
+        groups[s].insert(groups[s].end(), groups[t].begin(), groups[t].end());
+        for (int u = 0; u < n; u++) {
+            Wm[s][u] = Wm[s][u] + Wm[t][u];
+            Wm[u][s] = Wm[u][s] + Wm[u][t];
+        }
+        Wm[s][s] = W2{};
+        active.erase(std::find(active.begin(), active.end(), t));
+    }
+    std::sort(best_group.begin(), best_group.end());
+    return CutInfo{best_group, best.q, best.e, phases};
+}
+
+static void finish_plan(kf_pipeline *p, kf_plan *plan)
+{
+    for (auto &b : plan->blocks) std::sort(b.begin(), b.end());
+    std::sort(plan->blocks.begin(), plan->blocks.end(),
+              [](const std::vector<int> &a, const std::vector<int> &b) { return a.back() < b.back(); });
+    plan->beta_q = plan->beta_eps = 0;
+    for (auto &b : plan->blocks) {
+        std::set<int> S(b.begin(), b.end());
+        for (const EdgeInfo &e : plan->edges)
+            if (S.count(e.ks) && S.count(e.kd)) { plan->beta_q += e.q; plan->beta_eps += e.eps; }
+    }
+    for (auto &b : plan->blocks) plan->info.push_back(analyse_block(p, b));
+    // band halo: max accumulated vertical radius from an input to an output
+    std::vector<int> dist(p->n_images(), -1);
+    for (int o : p->outputs) dist[o] = 0;
+    for (int k = (int)p->ops.size() - 1; k >= 0; k--) {
+        int d = dist[p->n_inputs + k];
+        if (d < 0) d = 0;                // dead kernels still run
+        for (int img : p->ops[k].inputs) dist[img] = std::max(dist[img], d + p->ops[k].ry());
+    }
+    plan->halo_rows = 0;
+    for (int i = 0; i < p->n_inputs; i++) plan->halo_rows = std::max(plan->halo_rows, dist[i]);
+    plan->pipe = p;
+    p->frozen = true;
+}
+
+kf_plan *plan_fusion(kf_pipeline *p, const kf_model_params &m)
+{
+    if (p->ops.empty()) fail(KF_ERR_ARG, "pipeline has no kernels");
+    if (!(m.ts > 0) || m.tile_w <= 0 || m.tile_h <= 0 || !(m.c_mshared > 0))
+        fail(KF_ERR_ARG, "invalid model parameters");
+    auto plan = std::make_unique<kf_plan>();
+    plan->edges = edge_weights(p, m);                         // Alg. 1 lines 2-4
+    std::deque<std::vector<int>> Sp;                          // line 6
+    std::vector<int> all(p->ops.size());
+    for (size_t i = 0; i < all.size(); i++) all[i] = (int)i;
+    Sp.push_back(all);
+    while (!Sp.empty()) {                                     // lines 7-17
+        std::vector<int> blk = Sp.front();
+        Sp.pop_front();
+        std::set<int> S(blk.begin(), blk.end());
+        if (blk.size() == 1 || is_legal(p, S, m, plan->edges)) {
+            plan->blocks.push_back(blk);                      // line 10
+        } else {
+            CutInfo c = stoer_wagner(blk, plan->edges);       // line 13
+            std::vector<int> other;
+            std::set<int> side(c.side.begin(), c.side.end());
+            for (int k : blk)
+                if (!side.count(k)) other.push_back(k);
+            plan->cuts.push_back(c);
+            Sp.push_back(c.side);
+            Sp.push_back(other);
+        }
+    }
+    finish_plan(p, plan.get());
+    return plan.release();
+}
+
+kf_plan *plan_from_blocks(kf_pipeline *p, std::vector<std::vector<int>> blocks, bool check)
+{
+    auto plan = std::make_unique<kf_plan>();
+    kf_model_params m;
+    kf_model_params_paper(&m);
+    plan->edges = edge_weights(p, m);
+    for (auto &b : blocks) {
+        if (check && b.size() > 1) {
+            std::set<int> S(b.begin(), b.end());
+            if (!dependence_legal(p, S) || !header_legal(p, S)) {
+                std::string s;
+                for (int k : b) s += " " + std::to_string(k);
+                fail(KF_ERR_ILLEGAL_BLOCK, "block {" + s + " } is not legal (dependence/header)");
+            }
+        }
+    }
+    plan->blocks = std::move(blocks);
+    finish_plan(p, plan.get());
+    return plan.release();
+}
+
+// Block analysis: sink, external images, halos, staged kernels.
+BlockInfo analyse_block(const kf_pipeline *p, const std::vector<int> &kernels)
+{
+    BlockInfo b;
+    b.kernels = kernels;
+    std::sort(b.kernels.begin(), b.kernels.end());
+    std::set<int> S(b.kernels.begin(), b.kernels.end());
+    auto co = consumers(p);
+    for (int k : b.kernels) {
+        bool inner = false;
+        for (int c : co[k]) inner |= S.count(c) > 0;
+        if (!inner) b.sink = k;                 // legal blocks have exactly one
+    }
+    for (auto it = b.kernels.rbegin(); it != b.kernels.rend(); ++it) {
+        int k = *it;
+        int hx = 0, hy = 0;
+        for (int c : co[k])
+            if (S.count(c)) {
+                hx = std::max(hx, b.hx[c] + p->ops[c].rx());
+                hy = std::max(hy, b.hy[c] + p->ops[c].ry());
+                if (p->ops[c].kind == LOCAL) b.staged.insert(k);
+            }
+        b.hx[k] = hx;
+        b.hy[k] = hy;
+    }
+    std::set<int> ext;
+    for (int k : b.kernels)
+        for (int img : p->ops[k].inputs) {
+            bool inside = img >= p->n_inputs && S.count(img - p->n_inputs);
+            if (inside) continue;
+            ext.insert(img);
+            b.ext_hx[img] = std::max(b.ext_hx.count(img) ? b.ext_hx[img] : 0, b.hx[k] + p->ops[k].rx());
+            b.ext_hy[img] = std::max(b.ext_hy.count(img) ? b.ext_hy[img] : 0, b.hy[k] + p->ops[k].ry());
+        }
+    b.ext.assign(ext.begin(), ext.end());
+    for (int img : b.ext) {
+        b.Rx = std::max(b.Rx, b.ext_hx[img]);
+        b.Ry = std::max(b.Ry, b.ext_hy[img]);
+    }
+    int loc = 0, rep = 0;
+    for (int k : b.kernels)
+        if (p->ops[k].kind == LOCAL) { loc++; rep += p->ops[k].mode == KF_REPEAT; }
+    b.torus = loc > 0 && rep == loc;
+    return b;
+}
+
+}  // namespace kf

@@ -1,0 +1,359 @@
+// runtime.cu -- executor of libkfuse: compiles each partition block's
+// generated kernel with NVRTC for sm_100a (cached), loads it through the CUDA
+// driver API (entry points obtained from the runtime, so libkfuse.so loads on
+// a machine without a driver), owns the workspace of cut-edge images and
+// launches one kernel per block in topological order on the caller's stream
+// (Alg. 1 output: "each partition block in the ready set is fused into one
+// kernel").
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nvrtc.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
+#include <cstdio>
+#include <cstring>
+#include <fstream>
+#include <mutex>
+#include <sstream>
+
+#include "kf_internal.h"
+
+namespace kf {
+
+static const char *kDeviceHeader =
+#include "kf_device_cuh.inc"
+    ;
+
+// --------------------------------------------------------------- helpers
+#define KF_CUDA(call)                                                                         \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess)                                                                \
+            fail(KF_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_));            \
+    } while (0)
+
+struct Driver {
+    CUresult (*moduleLoadData)(CUmodule *, const void *) = nullptr;
+    CUresult (*moduleGetFunction)(CUfunction *, CUmodule, const char *) = nullptr;
+    CUresult (*moduleUnload)(CUmodule) = nullptr;
+    CUresult (*launchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
+                             CUstream, void **, void **) = nullptr;
+    CUresult (*getErrorString)(CUresult, const char **) = nullptr;
+};
+
+static Driver &driver()
+{
+    static Driver d;
+    static std::once_flag once;
+    static std::string err;
+    std::call_once(once, [] {
+        int ndev = 0;
+        cudaError_t e = cudaGetDeviceCount(&ndev);
+        if (e != cudaSuccess || ndev == 0) {
+            err = std::string("no CUDA device: ") + cudaGetErrorString(e);
+            return;
+        }
+        cudaFree(nullptr);   // initialise the primary context (shared with PyTorch)
+        auto get = [](const char *name, void **fn) {
+            cudaDriverEntryPointQueryResult q;
+            cudaError_t r = cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q);
+            if (r != cudaSuccess || q != cudaDriverEntryPointSuccess || !*fn)
+                err += std::string(" missing driver entry point ") + name;
+        };
+        get("cuModuleLoadData", (void **)&d.moduleLoadData);
+        get("cuModuleGetFunction", (void **)&d.moduleGetFunction);
+        get("cuModuleUnload", (void **)&d.moduleUnload);
+        get("cuLaunchKernel", (void **)&d.launchKernel);
+        get("cuGetErrorString", (void **)&d.getErrorString);
+    });
+    if (!err.empty() || !d.launchKernel) fail(KF_ERR_CUDA, "CUDA unavailable:" + err);
+    return d;
+}
+
+static void cu_check(CUresult r, const char *what)
+{
+    if (r == CUDA_SUCCESS) return;
+    const char *s = "unknown";
+    if (driver().getErrorString) driver().getErrorString(r, &s);
+    fail(KF_ERR_CUDA, std::string(what) + ": " + s);
+}
+
+static uint64_t fnv1a(const std::string &s, uint64_t h = 1469598103934665603ull)
+{
+    for (unsigned char c : s) { h ^= c; h *= 1099511628211ull; }
+    return h;
+}
+
+// Directory of the cubin cache: $KFUSE_CACHE_DIR, else <dir of libkfuse.so>/kcache.
+static std::string cache_dir()
+{
+    if (const char *e = getenv("KFUSE_CACHE_DIR")) return e;
+    Dl_info info;
+    if (dladdr((void *)&cache_dir, &info) && info.dli_fname) {
+        std::string f = info.dli_fname;
+        size_t pos = f.rfind('/');
+        if (pos != std::string::npos) return f.substr(0, pos) + "/kcache";
+    }
+    return "./kcache";
+}
+
+static const char *kNvrtcOpts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-DKF_NVRTC=1",
+                                   "--extra-device-vectorization"};
+
+// NVRTC -> sm_100a cubin, cached on disk by hash(source, header, options).
+static std::string compile_cubin(const std::string &src, const std::string &name)
+{
+    std::string key = src + kDeviceHeader;
+    for (const char *o : kNvrtcOpts) key += o;
+    char hex[32];
+    std::snprintf(hex, sizeof hex, "%016llx", (unsigned long long)fnv1a(key));
+    const std::string dir = cache_dir();
+    const std::string path = dir + "/" + name + "_" + hex + ".cubin";
+    {
+        std::ifstream f(path, std::ios::binary);
+        if (f) {
+            std::stringstream ss;
+            ss << f.rdbuf();
+            std::string s = ss.str();
+            if (s.size() > 16) return s;
+        }
+    }
+    nvrtcProgram prog;
+    const char *hdr_src[] = {kDeviceHeader};
+    const char *hdr_name[] = {"kf_device.cuh"};
+    if (nvrtcCreateProgram(&prog, src.c_str(), (name + ".cu").c_str(), 1, hdr_src, hdr_name) != NVRTC_SUCCESS)
+        fail(KF_ERR_NVRTC, "nvrtcCreateProgram failed");
+    nvrtcResult r = nvrtcCompileProgram(prog, (int)(sizeof kNvrtcOpts / sizeof kNvrtcOpts[0]), kNvrtcOpts);
+    if (r != NVRTC_SUCCESS) {
+        size_t n = 0;
+        nvrtcGetProgramLogSize(prog, &n);
+        std::string log(n, '\0');
+        nvrtcGetProgramLog(prog, &log[0]);
+        nvrtcDestroyProgram(&prog);
+        fail(KF_ERR_NVRTC, "NVRTC failed for " + name + ": " + log);
+    }
+    size_t n = 0;
+    nvrtcGetCUBINSize(prog, &n);
+    std::string cubin(n, '\0');
+    nvrtcGetCUBIN(prog, &cubin[0]);
+    nvrtcDestroyProgram(&prog);
+    mkdir(dir.c_str(), 0775);
+    std::string tmp = path + "." + std::to_string(getpid()) + ".tmp";
+    {
+        std::ofstream f(tmp, std::ios::binary);
+        if (f) f.write(cubin.data(), (std::streamsize)cubin.size());
+    }
+    if (rename(tmp.c_str(), path.c_str()) != 0) unlink(tmp.c_str());
+    return cubin;
+}
+
+struct CompiledBlock {
+    CUmodule mod = nullptr;
+    CUfunction fn = nullptr;
+    int tile_w = 32, tile_h = 8, threads = 256;
+    std::string source;
+    ~CompiledBlock()
+    {
+        if (mod && driver().moduleUnload) driver().moduleUnload(mod);
+    }
+};
+
+struct Runtime {
+    std::map<uint64_t, std::shared_ptr<CompiledBlock>> modules;   // by source hash
+    std::vector<void *> stage_in, stage_out;                      // kf_run_host staging
+    size_t stage_bytes = 0;
+    int device = -1;
+    ~Runtime()
+    {
+        for (void *q : stage_in) cudaFree(q);
+        for (void *q : stage_out) cudaFree(q);
+    }
+};
+
+// Compile-only path usable without a GPU (build() warms the in-tree cache).
+std::string compile_block_cubin(const kf_pipeline *p, const kf_plan *plan, int i)
+{
+    return compile_cubin(generate_block(p, plan->info[i], i, 0, 0), kernel_name(i));
+}
+
+void prepare(kf_pipeline *p, kf_plan *plan)
+{
+    if (plan->prepared) return;
+    Driver &d = driver();
+    if (!p->rt) p->rt = new Runtime();
+    int dev = 0;
+    KF_CUDA(cudaGetDevice(&dev));
+    if (p->rt->device >= 0 && p->rt->device != dev) fail(KF_ERR_CUDA, "pipeline used on two devices");
+    p->rt->device = dev;
+    plan->compiled.clear();
+    for (size_t i = 0; i < plan->blocks.size(); i++) {
+        std::string src = generate_block(p, plan->info[i], (int)i, 0, 0);
+        uint64_t h = fnv1a(src);
+        auto it = p->rt->modules.find(h);
+        if (it == p->rt->modules.end()) {
+            auto cb = std::make_shared<CompiledBlock>();
+            std::string cubin = compile_cubin(src, kernel_name((int)i));
+            cu_check(d.moduleLoadData(&cb->mod, cubin.data()), "cuModuleLoadData");
+            cu_check(d.moduleGetFunction(&cb->fn, cb->mod, kernel_name((int)i).c_str()), "cuModuleGetFunction");
+            cb->source = src;
+            it = p->rt->modules.emplace(h, cb).first;
+        }
+        plan->compiled.push_back(it->second);
+    }
+    // workspace: block sinks that are not marked outputs (cut edges), full height
+    std::set<int> outs(p->outputs.begin(), p->outputs.end());
+    for (auto &b : plan->info) {
+        int img = p->n_inputs + b.sink;
+        bool consumed = false;
+        for (auto &b2 : plan->info)
+            for (int e : b2.ext) consumed |= e == img;
+        if (!outs.count(img) || consumed) {
+            if (!plan->workspace.count(img)) {
+                void *q = nullptr;
+                if (cudaMalloc(&q, (size_t)p->W * p->H * 4) != cudaSuccess)
+                    fail(KF_ERR_OOM, "workspace allocation failed");
+                plan->workspace[img] = q;
+            }
+        }
+    }
+    plan->prepared = true;
+}
+
+// Executes rows [row0, row1) of every output.  Full-image run: row0 = 0,
+// row1 = H, inputs hold all rows (in_row0 = 0).  Band run: inputs hold rows
+// from in_row0; each block computes its sink over the rows its consumers need.
+void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
+         void *stream, int row0, int row1, int in_row0)
+{
+    if (n_in != p->n_inputs || (n_in && !din)) fail(KF_ERR_ARG, "wrong number of inputs");
+    if (n_out != (int)p->outputs.size() || (n_out && !dout)) fail(KF_ERR_ARG, "wrong number of outputs");
+    for (int i = 0; i < n_in; i++)
+        if (!din[i] || ((uintptr_t)din[i] & 15)) fail(KF_ERR_ARG, "input pointers must be non-null, 16-B aligned");
+    for (int j = 0; j < n_out; j++)
+        if (!dout[j] || ((uintptr_t)dout[j] & 15)) fail(KF_ERR_ARG, "output pointers must be non-null, 16-B aligned");
+    prepare(p, plan);
+    Driver &d = driver();
+    const bool band = !(row0 == 0 && row1 == p->H && in_row0 == 0);
+    const int nimg = p->n_images();
+    // rows each image must be available over
+    std::vector<int> lo(nimg, INT32_MAX), hi(nimg, INT32_MIN);
+    std::vector<int> blo(plan->blocks.size()), bhi(plan->blocks.size());
+    for (int o : p->outputs) { lo[o] = row0; hi[o] = row1; }
+    for (int bi = (int)plan->blocks.size() - 1; bi >= 0; bi--) {
+        const BlockInfo &b = plan->info[bi];
+        int s = p->n_inputs + b.sink;
+        if (lo[s] > hi[s]) { lo[s] = row0; hi[s] = row1; }      // dead kernel: same rows as outputs
+        blo[bi] = lo[s];
+        bhi[bi] = hi[s];
+        for (int e : b.ext) {
+            lo[e] = std::min(lo[e], std::max(0, lo[s] - b.ext_hy.at(e)));
+            hi[e] = std::max(hi[e], std::min(p->H, hi[s] + b.ext_hy.at(e)));
+        }
+    }
+    // where each image lives
+    std::vector<void *> ptr(nimg, nullptr);
+    std::vector<int> base(nimg, 0);
+    for (int i = 0; i < p->n_inputs; i++) { ptr[i] = const_cast<void *>(din[i]); base[i] = in_row0; }
+    for (auto &kv : plan->workspace) { ptr[kv.first] = kv.second; base[kv.first] = 0; }
+    std::vector<std::pair<int, int>> band_copies;   // (image, output slot) copied at the end
+    for (int j = 0; j < n_out; j++) {
+        int o = p->outputs[j];
+        if (plan->workspace.count(o) && band) {
+            band_copies.push_back({o, j});
+        } else {
+            ptr[o] = dout[j];
+            base[o] = band ? row0 : 0;
+        }
+    }
+    CUstream st = (CUstream)stream;
+    for (size_t bi = 0; bi < plan->blocks.size(); bi++) {
+        const BlockInfo &b = plan->info[bi];
+        const CompiledBlock &cb = *plan->compiled[bi];
+        struct Args {
+            const void *img[16];
+            int base[16];
+            void *out;
+            int out_base;
+            int W, H, r0, r1, tiles_x, tiles_y;
+        } a;
+        std::memset(&a, 0, sizeof a);
+        for (size_t s = 0; s < b.ext.size(); s++) {
+            a.img[s] = ptr[b.ext[s]];
+            a.base[s] = base[b.ext[s]];
+        }
+        int sink = p->n_inputs + b.sink;
+        a.out = ptr[sink];
+        a.out_base = base[sink];
+        a.W = p->W;
+        a.H = p->H;
+        a.r0 = blo[bi];
+        a.r1 = bhi[bi];
+        a.tiles_x = (p->W + cb.tile_w - 1) / cb.tile_w;
+        a.tiles_y = (a.r1 - a.r0 + cb.tile_h - 1) / cb.tile_h;
+        if (a.tiles_y <= 0) continue;
+        if (a.tiles_y > 65535) fail(KF_ERR_ARG, "image too tall for the v1 grid");
+        void *params[] = {&a};
+        cu_check(d.launchKernel(cb.fn, a.tiles_x, a.tiles_y, 1, cb.threads, 1, 1, 0, st, params, nullptr),
+                 "cuLaunchKernel");
+    }
+    for (auto &c : band_copies) {
+        const char *src = (const char *)plan->workspace[c.first] + (size_t)row0 * p->W * 4;
+        KF_CUDA(cudaMemcpyAsync(dout[c.second], src, (size_t)(row1 - row0) * p->W * 4, cudaMemcpyDeviceToDevice,
+                                (cudaStream_t)stream));
+    }
+}
+
+void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
+              void *stream)
+{
+    if (n_in != p->n_inputs || n_out != (int)p->outputs.size()) fail(KF_ERR_ARG, "wrong number of buffers");
+    prepare(p, plan);
+    Runtime &rt = *p->rt;
+    const size_t bytes = (size_t)p->W * p->H * 4;
+    if (rt.stage_bytes != bytes || rt.stage_in.size() != (size_t)n_in || rt.stage_out.size() != (size_t)n_out) {
+        for (void *q : rt.stage_in) cudaFree(q);
+        for (void *q : rt.stage_out) cudaFree(q);
+        rt.stage_in.assign(n_in, nullptr);
+        rt.stage_out.assign(n_out, nullptr);
+        for (auto &q : rt.stage_in)
+            if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
+        for (auto &q : rt.stage_out)
+            if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
+        rt.stage_bytes = bytes;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    for (int i = 0; i < n_in; i++) KF_CUDA(cudaMemcpyAsync(rt.stage_in[i], hin[i], bytes, cudaMemcpyHostToDevice, s));
+    std::vector<const void *> din(rt.stage_in.begin(), rt.stage_in.end());
+    run(p, plan, din.data(), n_in, rt.stage_out.data(), n_out, stream, 0, p->H, 0);
+    for (int j = 0; j < n_out; j++) KF_CUDA(cudaMemcpyAsync(hout[j], rt.stage_out[j], bytes, cudaMemcpyDeviceToHost, s));
+    KF_CUDA(cudaStreamSynchronize(s));
+}
+
+void release_plan(kf_plan *plan)
+{
+    for (auto &kv : plan->workspace) cudaFree(kv.second);
+    plan->workspace.clear();
+    plan->compiled.clear();
+}
+
+void release_runtime(kf_pipeline *p) { delete p->rt; p->rt = nullptr; }
+
+}  // namespace kf
+
+kf_pipeline::~kf_pipeline() { kf::release_runtime(this); }
+kf_plan::~kf_plan() { kf::release_plan(this); }
+
+// Compile-only entry point (no GPU needed): warms the cubin cache for every
+// block of a plan.  Used by __graft_entry__.build() and tests.
+extern "C" kf_status kf_compile_plan(kf_pipeline *p, const kf_plan *plan)
+{
+    try {
+        for (size_t i = 0; i < plan->blocks.size(); i++) kf::compile_block_cubin(p, plan, (int)i);
+        return KF_OK;
+    } catch (const kf::Error &e) {
+        kf::set_error(e.msg);
+        return e.st;
+    }
+}

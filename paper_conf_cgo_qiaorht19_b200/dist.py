@@ -1,0 +1,77 @@
+"""Row-band data parallelism across the GPUs of one node.
+
+GPU g owns output rows [g*H/P, (g+1)*H/P).  One fused plan needs R =
+plan.halo_rows input rows above and below its band (the accumulated vertical
+stencil radius); those rows live on the neighbours g-1 and g+1 and are
+exchanged with one point-to-point step per run (NCCL send/recv over
+NVLink/NVSwitch via torch.distributed; gloo on CPU for tests).  The fused
+kernels then run on the band through kf_run_band, applying border modes at the
+GLOBAL image edges, so the banded result is bit-identical to a single-GPU run.
+
+Plumbing only: the exchange is torch.distributed, the compute is libkfuse.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import torch
+import torch.distributed as dist
+
+
+@dataclass
+class Band:
+    rank: int
+    world: int
+    height: int         # global image height
+    halo: int           # R
+    row0: int           # owned output rows [row0, row1)
+    row1: int
+    in0: int            # rows held in the input buffer [in0, in1)
+    in1: int
+
+    @property
+    def rows(self) -> int:
+        return self.row1 - self.row0
+
+    @property
+    def top(self) -> int:          # halo rows above the band actually present
+        return self.row0 - self.in0
+
+    @property
+    def bottom(self) -> int:
+        return self.in1 - self.row1
+
+
+def partition(height: int, world: int, rank: int, halo: int) -> Band:
+    """Balanced contiguous row bands; the halo is clipped at the global edges."""
+    r0 = height * rank // world
+    r1 = height * (rank + 1) // world
+    if halo > r1 - r0 and world > 1:
+        raise ValueError(f"band of {r1 - r0} rows is thinner than the halo {halo}")
+    return Band(rank, world, height, halo, r0, r1, max(0, r0 - halo), min(height, r1 + halo))
+
+
+def exchange_halos(buf: torch.Tensor, band: Band, group=None) -> None:
+    """buf holds rows [in0, in1) of the global image (first dim = rows); the
+    owned rows [row0, row1) are valid.  Fills the top/bottom halo rows from the
+    neighbours: one batched send/recv step (no collective)."""
+    if band.world == 1 or band.halo == 0:
+        return
+    ops = []
+    t, b, n = band.top, band.bottom, band.rows
+    if band.rank > 0:
+        ops.append(dist.P2POp(dist.isend, buf[t:t + band.halo].contiguous(), band.rank - 1, group))
+        ops.append(dist.P2POp(dist.irecv, buf[0:t], band.rank - 1, group))
+    recv_bottom = None
+    if band.rank < band.world - 1:
+        ops.append(dist.P2POp(dist.isend, buf[t + n - band.halo:t + n].contiguous(), band.rank + 1, group))
+        recv_bottom = buf[t + n:t + n + b]
+        ops.append(dist.P2POp(dist.irecv, recv_bottom, band.rank + 1, group))
+    for req in dist.batch_isend_irecv(ops):
+        req.wait()
+
+
+def run_band(plan, band: Band, inputs, outputs, stream=None) -> None:
+    """inputs: device tensors holding rows [in0, in1) (halo exchanged);
+    outputs: device tensors of band.rows rows."""
+    plan.run_band(band.row0, band.row1, inputs, band.in0, band.in1, outputs, stream)

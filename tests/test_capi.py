@@ -1,0 +1,146 @@
+"""C-ABI on CPU (no GPU calls): the library loads and exports every symbol the
+header declares; the C++ planner agrees partition-for-partition with the
+reference planner (oracle/planner.py); argument validation; generated kernels
+compile with NVRTC for sm_100a."""
+import os
+import random
+import re
+
+import pytest
+
+from kf_inputs import pipelines as P
+from oracle import planner as PL
+from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_exports_every_declared_symbol():
+    with open(os.path.join(ROOT, "include", "kfuse.h")) as f:
+        hdr = f.read()
+    declared = set(re.findall(r"^\s*(?:[\w\s\*]+?)\b(kf_\w+)\s*\(", hdr, re.M))
+    assert len(declared) >= 28
+    for name in declared:
+        assert hasattr(K.lib, name), f"libkfuse.so does not export {name}"
+    assert declared <= set(K.EXPORTED), sorted(declared - set(K.EXPORTED))
+    assert "sm_100a" in K.version()
+
+
+def _ref_model(profile):
+    return PL.PAPER_PROFILE if profile == "paper" else PL.B200_PROFILE
+
+
+def _compare(spec, profile):
+    ref = PL.get_legal_partitions(spec, _ref_model(profile))
+    p = K.Pipeline.from_spec(spec)
+    plan = p.plan_fusion(profile)
+    assert plan.blocks == ref.blocks
+    assert plan.objective == ref.beta
+    assert [(c[0], c[1], c[2]) for c in plan.cuts] == [(c[1], c[2], c[3]) for c in ref.cuts]
+    for (ks, kd), e in ref.info.items():
+        got = plan.edge(ks, kd)
+        assert got["w"] == e.w and got["ctx_legal"] == e.ctx_legal and got["profitable"] == e.profitable
+        assert got["is_eps"] == (e.weight[1] == 1)
+    return plan
+
+
+@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10"])
+@pytest.mark.parametrize("profile", ["paper", "b200"])
+def test_planner_matches_reference_on_workloads(wl, profile):
+    _compare(P.WORKLOADS[wl](64, 64), profile)
+
+
+def test_harris_plan_pins_through_the_abi():
+    """Fig. 3 through the C-ABI: 6 blocks, beta 912, first cut {sy,gy} at 2 eps after 8 phases."""
+    plan = _compare(P.harris(256, 256), "paper")
+    assert plan.num_launches == 6 and plan.objective == (912 << 20, 0)
+    assert plan.cuts[0] == ([3, 6], (0, 2), 8)
+    assert plan.halo_rows == 2
+
+
+@pytest.mark.parametrize("seed", range(80))
+def test_planner_matches_reference_on_random_dags(seed):
+    rng = random.Random(5000 + seed)
+    spec = P.random_pipeline(rng, 16, 16, rng.choice(["f32", "u8x4"]), rng.randint(1, 9))
+    _compare(spec, rng.choice(["paper", "b200"]))
+
+
+def test_unfused_and_from_blocks():
+    spec = P.harris(32, 32)
+    p = K.Pipeline.from_spec(spec)
+    assert p.plan_unfused().blocks == [[k] for k in range(9)]
+    p2 = K.Pipeline.from_spec(spec)
+    plan = p2.plan_from_blocks([0, 1, 2, 3, 4, 2, 3, 4, 5])
+    assert plan.blocks == [[0], [1], [2, 5], [3, 6], [4, 7], [8]]
+    p3 = K.Pipeline.from_spec(spec)
+    with pytest.raises(K.KfError) as e:
+        p3.plan_from_blocks([0, 0, 1, 2, 3, 4, 5, 6, 7])     # {dx, dy}: two sinks
+    assert e.value.name == "KF_ERR_ILLEGAL_BLOCK"
+    p4 = K.Pipeline.from_spec(spec)
+    with pytest.raises(K.KfError):
+        p4.plan_from_blocks([0, 1, 0, 3, 4, 5, 6, 7, 8])     # {dx, sx}: external output (Fig. 2c)
+    p5 = K.Pipeline.from_spec(spec)
+    assert len(p5.plan_from_blocks([0] * 9).blocks) == 1    # whole DAG is dependence-legal
+
+
+def test_argument_validation():
+    p = K.Pipeline(8, 8, "f32")
+    i = p.add_input()
+    with pytest.raises(K.KfError) as e:
+        p.add_point_op([i + 5], [P.L(0)])
+    assert e.value.name == "KF_ERR_BAD_ID"
+    with pytest.raises(K.KfError) as e:
+        p.add_point_op([i], [P.L(0), P.ADD])
+    assert e.value.name == "KF_ERR_PROGRAM"
+    with pytest.raises(K.KfError) as e:
+        p.add_point_op([i], [P.L(0), P.SHR(1)])              # integer op in a float pipeline
+    assert e.value.name == "KF_ERR_PROGRAM"
+    with pytest.raises(K.KfError) as e:
+        p.add_local_op(i, [[1, 1]], "clamp")                   # even mask
+    assert e.value.name == "KF_ERR_MASK"
+    a = p.add_local_op(i, [[1, 2, 1]], "mirror")
+    p.mark_output(a)
+    with pytest.raises(K.KfError):
+        p.mark_output(a)
+    p.plan_unfused()
+    with pytest.raises(K.KfError) as e:
+        p.add_point_op([a], [P.L(0)])
+    assert e.value.name == "KF_ERR_FROZEN"
+    q = K.Pipeline(8, 8, "u8x4")
+    j = q.add_input()
+    with pytest.raises(K.KfError) as e:
+        q.add_local_op(j, [[0.5, 1, 0.5]], "clamp")
+    assert e.value.name == "KF_ERR_MASK"
+    with pytest.raises(K.KfError):
+        q.add_local_op(j, [[1, 1, 1]], "constant", constant=300)
+    with pytest.raises(K.KfError):
+        K.Pipeline(0, 5, "f32")
+
+
+def test_repeat_mixing_is_not_fused():
+    """Reading R-8: a fused block's local kernels all use REPEAT or none does."""
+    p = P.Pipeline("mix", 16, 16, "f32")
+    i = p.input()
+    a = p.local("a", i, P.GAUSS3_N, "repeat")
+    b = p.local("b", a, P.GAUSS3_N, "clamp")
+    p.output(b)
+    spec = p.spec()
+    plan = K.Pipeline.from_spec(spec).plan_fusion("b200")
+    assert plan.blocks == [[0], [1]]
+    with pytest.raises(K.KfError):
+        K.Pipeline.from_spec(spec).plan_from_blocks([0, 0])
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_generated_kernels_compile_for_sm100a(seed, tmp_path, monkeypatch):
+    """Every block of random plans compiles with NVRTC to an sm_100a cubin."""
+    monkeypatch.setenv("KFUSE_CACHE_DIR", str(tmp_path))
+    rng = random.Random(9000 + seed)
+    spec = P.random_pipeline(rng, 20, 12, rng.choice(["f32", "u8x4"]), rng.randint(2, 7))
+    p = K.Pipeline.from_spec(spec)
+    plan = p.plan_fusion(rng.choice(["paper", "b200"]))
+    plan.compile()
+    cubins = list(tmp_path.glob("*.cubin"))
+    assert len(cubins) == len(plan.blocks)
+    blob = cubins[0].read_bytes()
+    assert blob[:4] == b"\x7fELF"

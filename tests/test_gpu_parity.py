@@ -1,0 +1,205 @@
+"""GPU parity: the fused sm_100a kernels (through the C-ABI) against the unfused
+CPU oracle on the same seeded inputs.
+
+Bar: u8x4 pipelines bit-exact; f32 pipelines
+max|gpu - oracle| / max|oracle| <= 1e-5 (the oracle is fp64, the GPU f32).
+"""
+import random
+
+import numpy as np
+import pytest
+import torch
+
+from kf_inputs import gen
+from kf_inputs import pipelines as P
+from oracle import oracle as O
+from oracle import planner as PL
+from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-5
+
+
+def _inputs(spec, seed):
+    return [gen.image(spec["dtype"], seed + 101 * j, spec["width"], spec["height"]) for j in range(spec["n_inputs"])]
+
+
+def _alloc(spec):
+    H, W = spec["height"], spec["width"]
+    dt = torch.float32 if spec["dtype"] == "f32" else torch.uint8
+    shape = (H, W) if spec["dtype"] == "f32" else (H, W, 4)
+    return [torch.empty(shape, dtype=dt, device="cuda") for _ in spec["outputs"]]
+
+
+def make_plan(spec, kind):
+    p = K.Pipeline.from_spec(spec)
+    if kind == "unfused":
+        return p.plan_unfused()
+    if kind == "whole":
+        return p.plan_from_blocks([0] * len(spec["ops"]))
+    return p.plan_fusion(kind)
+
+
+def run_gpu(spec, plan, ins):
+    d_in = [torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in ins]
+    outs = _alloc(spec)
+    plan.run(d_in, outs)
+    torch.cuda.synchronize()
+    return [o.cpu().numpy() for o in outs]
+
+
+def check(spec, got, ref, what=""):
+    if spec["dtype"] == "u8x4":
+        bad = np.argwhere(np.any(got != ref, axis=-1))
+        assert len(bad) == 0, f"{what}: {len(bad)} pixels differ, first {bad[:5].tolist()}"
+        return 0.0
+    got = got.astype(np.float64)
+    scale = np.abs(ref).max()
+    err = np.abs(got - ref).max() / (scale if scale > 0 else 1.0)
+    assert np.all(np.isfinite(got)) == np.all(np.isfinite(ref))
+    assert err <= TOL, f"{what}: normalised error {err:.3g} > {TOL}"
+    return err
+
+
+def parity(spec, kind, seed=1):
+    ins = _inputs(spec, seed)
+    plan = make_plan(spec, kind)
+    got = run_gpu(spec, plan, ins)
+    ref = O.run(spec, ins)
+    for g, o in zip(got, spec["outputs"]):
+        check(spec, g, ref[o], f"{spec['name']} {kind} {spec['width']}x{spec['height']}")
+    return plan
+
+
+# --------------------------------------------------------------- workloads
+
+@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10"])
+@pytest.mark.parametrize("kind", ["unfused", "paper", "b200"])
+@pytest.mark.parametrize("size", [(67, 41), (256, 256)])
+def test_workloads(wl, kind, size):
+    parity(P.WORKLOADS[wl](*size), kind)
+
+
+@pytest.mark.parametrize("mode", P.MODES)
+@pytest.mark.parametrize("wl", ["harris", "deep10"])
+def test_workloads_all_border_modes_fused(wl, mode):
+    """Index exchange under every border mode (pad-once differs under
+    clamp/constant for Harris and under every non-wrap mode for deep10)."""
+    spec = P.WORKLOADS[wl](45, 37, mode=mode)
+    plan = parity(spec, "b200")
+    if mode != "repeat" or wl == "deep10":
+        assert plan.num_launches == 1
+
+
+def test_fig4_fused_on_gpu():
+    """Fig. 4c through the fused GPU kernel: 763 at (0,0), 992 at (2,2)."""
+    spec = P.fig4("clamp")
+    img = np.array(P.FIG4_IMAGE, np.float32)
+    plan = make_plan(spec, "whole")
+    assert plan.num_launches == 1
+    out = run_gpu(spec, plan, [img])[0]
+    assert out[0, 0] == 763 and out[2, 2] == 992
+    ref = O.run(spec, [img])[2]
+    np.testing.assert_array_equal(out, ref)
+
+
+@pytest.mark.parametrize("size", [(1, 1), (2, 3), (3, 2), (5, 5), (31, 9), (33, 17), (7, 70)])
+@pytest.mark.parametrize("wl", ["harris", "deep10", "unsharp"])
+def test_tiny_and_ragged_images(wl, size):
+    """Images smaller than the halo (mirror folds repeatedly), ragged tiles."""
+    for mode in ("clamp", "mirror", "mirror101", "constant", "repeat"):
+        parity(P.WORKLOADS[wl](*size, mode=mode), "b200")
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_random_dags(seed):
+    rng = random.Random(70000 + seed)
+    dtype = rng.choice(["f32", "u8x4"])
+    W, H = rng.choice([(1, 1), (4, 3), (9, 9), (33, 17), (70, 45), (129, 20)])
+    spec = P.random_pipeline(rng, W, H, dtype, rng.randint(2, 8))
+    for kind in ("unfused", "paper", "b200"):
+        parity(spec, kind, seed)
+    # the exhaustive optimum's partition as well (any legal partition must be exact)
+    best, blocks = PL.brute_force(spec, PL.B200_PROFILE) if len(spec["ops"]) <= 7 else (None, None)
+    if blocks:
+        lab = [0] * len(spec["ops"])
+        for b, ks in enumerate(blocks):
+            for k in ks:
+                lab[k] = b
+        ins = _inputs(spec, seed)
+        plan = K.Pipeline.from_spec(spec).plan_from_blocks(lab)
+        got = run_gpu(spec, plan, ins)
+        ref = O.run(spec, ins)
+        for g, o in zip(got, spec["outputs"]):
+            check(spec, g, ref[o], "brute-force partition")
+
+
+# ------------------------------------------------------ full BASELINE sizes
+
+def _sample_points(W, H, rng, n=1500):
+    ys = list(rng.integers(0, H, n)) + [0, 0, H - 1, H - 1] + [0] * 20 + [H - 1] * 20 + list(range(min(H, 8)))
+    xs = list(rng.integers(0, W, n)) + [0, W - 1, 0, W - 1] + list(rng.integers(0, W, 40)) + [0] * min(H, 8)
+    return np.array(ys), np.array(xs)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3", "C3s", "C4"])
+def test_full_size_sampled(cfg):
+    """At BASELINE.json's full sizes, in the launch configuration bench.py times
+    (B200-profile plan): sampled outputs against the recursive oracle, and the
+    fused result against the unfused GPU run element by element."""
+    spec, seed = P.config(cfg)
+    ins = _inputs(spec, seed)
+    fused = make_plan(spec, "b200")
+    got = run_gpu(spec, fused, ins)[0]
+    rng = np.random.default_rng(3)
+    ys, xs = _sample_points(spec["width"], spec["height"], rng)
+    ref = O.eval_points(spec, ins, spec["outputs"][0], ys, xs)
+    if spec["dtype"] == "u8x4":
+        np.testing.assert_array_equal(got[ys, xs], ref)
+    else:
+        scale = np.abs(ref).max()
+        assert np.abs(got[ys, xs].astype(np.float64) - ref).max() / scale <= TOL
+    unf = run_gpu(spec, make_plan(spec, "unfused"), ins)[0]
+    if spec["dtype"] == "u8x4":
+        np.testing.assert_array_equal(got, unf)
+    else:
+        d = np.abs(got.astype(np.float64) - unf.astype(np.float64)).max() / np.abs(unf).max()
+        assert d <= TOL
+
+
+# ---------------------------------------------------------- other entry points
+
+def test_run_host_equals_run():
+    spec = P.harris(300, 200)
+    ins = _inputs(spec, 4)
+    plan = make_plan(spec, "b200")
+    dev = run_gpu(spec, plan, ins)[0]
+    out = np.empty_like(dev)
+    plan.run_host([np.ascontiguousarray(ins[0])], [out])
+    np.testing.assert_array_equal(out, dev)
+
+
+@pytest.mark.parametrize("wl", ["harris", "deep10", "unsharp"])
+@pytest.mark.parametrize("kind", ["unfused", "paper", "b200"])
+def test_bands_bit_identical(wl, kind):
+    """Row bands (the multi-GPU decomposition, §8(e)) reproduce the full run bit for bit."""
+    spec = P.WORKLOADS[wl](130, 97)
+    ins = _inputs(spec, 8)
+    plan = make_plan(spec, kind)
+    full = run_gpu(spec, plan, ins)[0]
+    H, R = spec["height"], plan.halo_rows
+    cuts = [0, 13, 40, 41, 97]
+    for r0, r1 in zip(cuts[:-1], cuts[1:]):
+        a0, a1 = max(0, r0 - R), min(H, r1 + R)
+        d_in = [torch.from_numpy(np.ascontiguousarray(x[a0:a1])).cuda() for x in ins]
+        out = torch.empty((r1 - r0,) + full.shape[1:], dtype=torch.float32 if spec["dtype"] == "f32" else torch.uint8,
+                          device="cuda")
+        plan.run_band(r0, r1, d_in, a0, a1, [out])
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(out.cpu().numpy(), full[r0:r1])
+
+
+def test_launch_count_matches_blocks():
+    spec = P.harris(512, 512)
+    for kind, n in (("unfused", 9), ("paper", 6), ("b200", 1)):
+        assert make_plan(spec, kind).num_launches == n
