@@ -291,7 +291,7 @@ kf_status kf_plan_kernel_source(kf_pipeline *p, const kf_plan *plan, int32_t blo
     return guard([&] {
         if (!p || !plan || plan->pipe != p) fail(KF_ERR_ARG, "plan does not belong to pipeline");
         if (block < 0 || block >= (int)plan->blocks.size()) fail(KF_ERR_ARG, "block index out of range");
-        std::string s = generate_block(p, plan->info[block], block, 0, 0);
+        std::string s = generate_block(p, plan->info[block], block);
         if (len) *len = s.size();
         if (buf && cap) {
             size_t n = std::min(cap - 1, s.size());
@@ -314,7 +314,7 @@ kf_status kf_run(kf_pipeline *p, const kf_plan *plan, const void *const *d_input
 {
     return guard([&] {
         if (!p || !plan || plan->pipe != p) fail(KF_ERR_ARG, "plan does not belong to pipeline");
-        run(p, const_cast<kf_plan *>(plan), d_inputs, n_in, d_outputs, n_out, stream, 0, p->H, 0);
+        run(p, const_cast<kf_plan *>(plan), d_inputs, n_in, d_outputs, n_out, stream, 0, p->H, 0, p->H);
     });
 }
 
@@ -342,7 +342,7 @@ kf_status kf_run_band(kf_pipeline *p, const kf_plan *plan, int32_t row0, int32_t
             if (op.kind == LOCAL && op.mode == KF_REPEAT)
                 fail(KF_ERR_ARG, "REPEAT border mode is not supported in band mode (needs a ring exchange)");
         run(p, const_cast<kf_plan *>(plan), d_in_band, p->n_inputs, d_out_band, (int)p->outputs.size(), stream,
-            row0, row1, in_row0);
+            row0, row1, in_row0, in_row1);
     });
 }
 

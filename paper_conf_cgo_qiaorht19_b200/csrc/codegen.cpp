@@ -3,21 +3,32 @@
 // Fusion techniques of the paper, B200 re-design:
 //   * point-based fusion: the producer body is inlined and the intermediate
 //     lives in a register (Listing 1 :225-252);
-//   * point-to-local / local-to-local: a producer consumed by an in-block local
-//     kernel ("staged") is computed ONCE per position of the tile plus its halo
-//     into shared memory; only the halo is recomputed by neighbouring tiles
-//     (instead of the paper's per-tap recompute);
-//   * border fusion + index exchange (§IV): staged values
-//     are indexed by in-image coordinates; a local consumer remaps an
-//     out-of-image tap with ITS OWN border mode before reading, so the fused
-//     result equals "clamp+conv+clamp+conv" (Fig. 4c), never "pad once".
-//     Tiles whose whole footprint is inside the image (the interior region,
-//     PAPER.md:1089-1093) run a variant without any remapping.
-//   * blocks whose local kernels all use REPEAT use a torus slot model: slot p
-//     holds the value at p mod n, which is exact because wrap needs no exchange.
+//   * point-to-local / local-to-local: the producer is computed once per pixel
+//     of the consumer's footprint and kept on chip; only the halo is
+//     recomputed by neighbouring tiles (instead of the paper's per-tap
+//     recompute);
+//   * the image is split into the paper's interior and border regions
+//     (§IV-B):
+//       - INTERIOR (fast path): every output pixel whose whole input footprint
+//         is inside the image.  One warp streams a 4-pixel-wide column chunk
+//         down a strip of rows: each kernel of the block is evaluated once per
+//         (row, pixel) in registers, vertical taps read per-image register
+//         ring buffers of past rows, horizontal taps come from the lane's own
+//         registers or warp shuffles, separable (rank-1) masks run
+//         vertical-then-horizontal.  No border logic at all.
+//       - BORDER FRAME (slow path): 2-D tiles whose producers are staged in
+//         shared memory over tile + halo.  Border fusion + index exchange
+//         (PAPER.md:1061-1133): staged values are indexed by in-image
+//         coordinates; a local consumer remaps an out-of-image tap with ITS OWN
+//         border mode before reading, so the fused result equals
+//         "clamp+conv+clamp+conv" (Fig. 4c), never "pad once".
+//   * blocks whose local kernels all use REPEAT use a torus slot model in the
+//     frame: slot p holds the value at p mod n (wrap needs no exchange).
 #include <algorithm>
+#include <cmath>
 #include <cstdio>
 #include <functional>
+#include <numeric>
 #include <sstream>
 
 #include "kf_internal.h"
@@ -37,122 +48,24 @@ std::string fconst(double v)
     return s;
 }
 
-struct Gen {
-    const kf_pipeline *p;
-    const BlockInfo &b;
-    int block;
-    int TW, TH;
+std::string iconst(long long v)
+{
+    if (v < 0) return "(" + std::to_string(v) + ")";
+    return std::to_string(v);
+}
+
+// postfix op-IR -> straight-line code, shared by both paths.  `loads` are the
+// values of LOAD k (a local op's post program: LOAD 0 = the accumulator).
+struct ProgEmitter {
     bool f32;
-    std::map<int, int> slot;             // external image -> slot
-    std::vector<std::vector<int>> groups;  // staged kernels grouped by halo, topological
-    std::ostringstream o;
-    int tmp = 0;
-
-    Gen(const kf_pipeline *p_, const BlockInfo &b_, int block_, int tw, int th)
-        : p(p_), b(b_), block(block_), TW(tw), TH(th), f32(p_->dtype == KF_F32) {}
-
+    int block;
+    int *tmp;
     std::string KV() const { return f32 ? "float" : "I4"; }
-    std::string var() { return "v" + std::to_string(tmp++); }
-    bool in_block(int img) const
-    {
-        return img >= p->n_inputs && std::binary_search(b.kernels.begin(), b.kernels.end(), img - p->n_inputs);
-    }
-    std::string smem_name(int k) const { return "s_" + std::to_string(k); }
-    int RW(int k) const { return TW + 2 * b.hx.at(k); }
-    int RH(int k) const { return TH + 2 * b.hy.at(k); }
+    std::string var() { return "v" + std::to_string((*tmp)++); }
 
-    // global load of an external image at in-image (or, torus: wrapped) coordinates
-    std::string ext_load(int img, const std::string &Y, const std::string &X) const
-    {
-        int s = slot.at(img);
-        return std::string(f32 ? "kf_ldf" : "kf_ldi") + "(a.img[" + std::to_string(s) + "], a.base[" +
-               std::to_string(s) + "], W, " + Y + ", " + X + ")";
-    }
-    std::string smem_load(int k, const std::string &Y, const std::string &X) const
-    {
-        std::string idx = "((" + Y + ") - (oy - " + std::to_string(b.hy.at(k)) + ")) * " + std::to_string(RW(k)) +
-                          " + ((" + X + ") - (ox - " + std::to_string(b.hx.at(k)) + "))";
-        return f32 ? smem_name(k) + "[" + idx + "]" : "kf_unpack(" + smem_name(k) + "[" + idx + "])";
-    }
-
-    // Emits code computing kernel/image `img` at position (y, x); returns the variable.
-    // memo: values already computed at this position; group: staged kernels computed
-    // in the current loop (read from memo, not smem).
-    std::string eval(int img, std::map<int, std::string> &memo, const std::set<int> &group, bool border,
+    std::string emit(std::ostringstream &o, const Op &op, int k, const std::vector<std::string> &loads,
                      const std::string &ind)
     {
-        auto it = memo.find(img);
-        if (it != memo.end()) return it->second;
-        std::string v = var();
-        if (!in_block(img)) {
-            std::string Y = "y", X = "x";
-            if (border && b.torus) { Y = "kf_wrap(y, H)"; X = "kf_wrap(x, W)"; }
-            o << ind << "const " << KV() << " " << v << " = " << ext_load(img, Y, X) << ";\n";
-            memo[img] = v;
-            return v;
-        }
-        int k = img - p->n_inputs;
-        if (b.staged.count(k) && !group.count(k)) {
-            o << ind << "const " << KV() << " " << v << " = " << smem_load(k, "y", "x") << ";\n";
-            memo[img] = v;
-            return v;
-        }
-        const Op &op = p->ops[k];
-        std::vector<std::string> loads;
-        std::string acc;
-        if (op.kind == POINT) {
-            for (int in : op.inputs) loads.push_back(eval(in, memo, group, border, ind));
-        } else {
-            acc = var();
-            o << ind << KV() << " " << acc << " = " << (f32 ? "0.0f" : "kf_i4(0)") << ";\n";
-            const int in = op.inputs[0];
-            const bool staged_in = in_block(in);
-            const int cy = op.mh / 2, cx = op.mw / 2;
-            for (int j = 0; j < op.mh; j++)
-                for (int i = 0; i < op.mw; i++) {
-                    double m = op.mask[(size_t)j * op.mw + i];
-                    if (m == 0.0) continue;
-                    const int dy = j - cy, dx = i - cx;
-                    std::string Y = "y + (" + std::to_string(dy) + ")", X = "x + (" + std::to_string(dx) + ")";
-                    std::string val;
-                    if (!border || (b.torus && staged_in)) {
-                        val = staged_in ? smem_load(in - p->n_inputs, Y, X) : ext_load(in, Y, X);
-                    } else if (b.torus) {
-                        val = ext_load(in, "kf_wrap(" + Y + ", H)", "kf_wrap(" + X + ", W)");
-                    } else {
-                        // index exchange: remap with THIS (consumer) kernel's border mode
-                        std::string mode = std::to_string(op.mode);
-                        std::string yy = var(), xx = var();
-                        o << ind << "const int " << yy << " = kf_border<" << mode << ">(" << Y << ", H);\n";
-                        o << ind << "const int " << xx << " = kf_border<" << mode << ">(" << X << ", W);\n";
-                        std::string rd = staged_in ? smem_load(in - p->n_inputs, yy, xx) : ext_load(in, yy, xx);
-                        if (op.mode == KF_CONSTANT) {
-                            std::string c = f32 ? fconst(op.constant) : "kf_i4(" + std::to_string((int)op.constant) + ")";
-                            val = "((" + yy + " < 0 || " + xx + " < 0) ? " + c + " : " + rd + ")";
-                        } else {
-                            val = rd;
-                        }
-                    }
-                    std::string mc = f32 ? fconst(m) : std::to_string((long long)m);
-                    o << ind << acc << " = kf_mac(" << acc << ", " << mc << ", " << val << ");\n";
-                }
-            loads.push_back(acc);
-        }
-        std::string r = program(op, k, loads, ind, op.kind == LOCAL && op.prog.empty() ? acc : "");
-        if (!f32) {
-            o << ind << "const I4 " << v << " = kf_satu8(" << r << ");\n";   // narrowing at the kernel boundary
-        } else {
-            o << ind << "const float " << v << " = " << r << ";\n";
-        }
-        memo[img] = v;
-        return v;
-    }
-
-    // postfix op-IR -> straight-line code; returns the result expression
-    std::string program(const Op &op, int k, const std::vector<std::string> &loads, const std::string &ind,
-                        const std::string &identity)
-    {
-        if (!identity.empty()) return identity;
         std::vector<std::string> st;
         auto pop = [&] { std::string s = st.back(); st.pop_back(); return s; };
         for (const Instr &in : op.prog) {
@@ -160,7 +73,7 @@ struct Gen {
             switch (in.op) {
             case KF_OP_LOAD: st.push_back(loads[op.kind == LOCAL ? 0 : in.arg]); continue;
             case KF_OP_CONST:
-                e = f32 ? fconst(in.imm) : "kf_i4(" + std::to_string((long long)(int64_t)in.imm) + ")";
+                e = f32 ? fconst(in.imm) : "kf_i4(" + iconst((long long)(int64_t)in.imm) + ")";
                 break;
             case KF_OP_ADD: case KF_OP_SUB: case KF_OP_MUL: case KF_OP_DIV: case KF_OP_MIN: case KF_OP_MAX:
             case KF_OP_POW: {
@@ -200,12 +113,127 @@ struct Gen {
         }
         return st.back();
     }
+};
 
-    void body(bool border)
+// ====================================================================== frame
+// Slow path: 2-D tiles with shared-memory staging and index exchange.  Used
+// for every output pixel outside the interior rectangle (and for the whole
+// image when the interior is empty).
+struct FrameGen {
+    const kf_pipeline *p;
+    const BlockInfo &b;
+    int block;
+    bool f32;
+    std::map<int, int> slot;               // external image -> slot
+    std::vector<std::vector<int>> groups;  // staged kernels grouped by halo, topological
+    std::ostringstream &o;
+    int tmp = 0;
+    int TW = 32, TH = 8;
+    ProgEmitter pe;
+
+    FrameGen(const kf_pipeline *p_, const BlockInfo &b_, int block_, std::ostringstream &o_)
+        : p(p_), b(b_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp} {}
+
+    std::string KV() const { return f32 ? "float" : "I4"; }
+    std::string var() { return "v" + std::to_string(tmp++); }
+    bool in_block(int img) const
+    {
+        return img >= p->n_inputs && std::binary_search(b.kernels.begin(), b.kernels.end(), img - p->n_inputs);
+    }
+    std::string smem_name(int k) const { return "s_" + std::to_string(k); }
+    int RW(int k) const { return TW + 2 * b.hx.at(k); }
+    int RH(int k) const { return TH + 2 * b.hy.at(k); }
+
+    std::string ext_load(int img, const std::string &Y, const std::string &X) const
+    {
+        int s = slot.at(img);
+        return std::string(f32 ? "kf_ldf" : "kf_ldi") + "(a.img[" + std::to_string(s) + "], a.base[" +
+               std::to_string(s) + "], W, " + Y + ", " + X + ")";
+    }
+    std::string smem_load(int k, const std::string &Y, const std::string &X) const
+    {
+        std::string idx = "((" + Y + ") - (oy - " + std::to_string(b.hy.at(k)) + ")) * " + std::to_string(RW(k)) +
+                          " + ((" + X + ") - (ox - " + std::to_string(b.hx.at(k)) + "))";
+        return f32 ? smem_name(k) + "[" + idx + "]" : "kf_unpack(" + smem_name(k) + "[" + idx + "])";
+    }
+
+    // Emits code computing image `img` at (y, x); returns the variable.
+    std::string eval(int img, std::map<int, std::string> &memo, const std::set<int> &group, const std::string &ind)
+    {
+        auto it = memo.find(img);
+        if (it != memo.end()) return it->second;
+        std::string v = var();
+        if (!in_block(img)) {
+            std::string Y = "y", X = "x";
+            if (b.torus) { Y = "kf_wrap(y, H)"; X = "kf_wrap(x, W)"; }
+            o << ind << "const " << KV() << " " << v << " = " << ext_load(img, Y, X) << ";\n";
+            memo[img] = v;
+            return v;
+        }
+        int k = img - p->n_inputs;
+        if (b.staged.count(k) && !group.count(k)) {
+            o << ind << "const " << KV() << " " << v << " = " << smem_load(k, "y", "x") << ";\n";
+            memo[img] = v;
+            return v;
+        }
+        const Op &op = p->ops[k];
+        std::vector<std::string> loads;
+        std::string acc;
+        if (op.kind == POINT) {
+            for (int in : op.inputs) loads.push_back(eval(in, memo, group, ind));
+        } else {
+            acc = var();
+            o << ind << KV() << " " << acc << " = " << (f32 ? "0.0f" : "kf_i4(0)") << ";\n";
+            const int in = op.inputs[0];
+            const bool staged_in = in_block(in);
+            const int cy = op.mh / 2, cx = op.mw / 2;
+            for (int j = 0; j < op.mh; j++)
+                for (int i = 0; i < op.mw; i++) {
+                    double m = op.mask[(size_t)j * op.mw + i];
+                    if (m == 0.0) continue;
+                    const int dy = j - cy, dx = i - cx;
+                    std::string Y = "y + (" + std::to_string(dy) + ")", X = "x + (" + std::to_string(dx) + ")";
+                    std::string val;
+                    if (b.torus && staged_in) {
+                        val = smem_load(in - p->n_inputs, Y, X);
+                    } else if (b.torus) {
+                        val = ext_load(in, "kf_wrap(" + Y + ", H)", "kf_wrap(" + X + ", W)");
+                    } else {
+                        // index exchange: remap with THIS (consumer) kernel's border mode
+                        std::string mode = std::to_string(op.mode);
+                        std::string yy = var(), xx = var();
+                        o << ind << "const int " << yy << " = kf_border<" << mode << ">(" << Y << ", H);\n";
+                        o << ind << "const int " << xx << " = kf_border<" << mode << ">(" << X << ", W);\n";
+                        std::string rd = staged_in ? smem_load(in - p->n_inputs, yy, xx) : ext_load(in, yy, xx);
+                        if (op.mode == KF_CONSTANT) {
+                            std::string c = f32 ? fconst(op.constant) : "kf_i4(" + iconst((int)op.constant) + ")";
+                            val = "((" + yy + " < 0 || " + xx + " < 0) ? " + c + " : " + rd + ")";
+                        } else {
+                            val = rd;
+                        }
+                    }
+                    std::string mc = f32 ? fconst(m) : iconst((long long)m);
+                    o << ind << acc << " = kf_mac(" << acc << ", " << mc << ", " << val << ");\n";
+                }
+            loads.push_back(acc);
+        }
+        std::string r = (op.kind == LOCAL && op.prog.empty()) ? acc : pe.emit(o, op, k, loads, ind);
+        if (!f32) {
+            o << ind << "const I4 " << v << " = kf_satu8(" << r << ");\n";   // narrowing at the kernel boundary
+        } else {
+            o << ind << "const float " << v << " = " << r << ";\n";
+        }
+        memo[img] = v;
+        return v;
+    }
+
+    // One tile shape: stage every staged kernel over tile + halo, then the sink
+    // over the tile, writing only pixels inside the frame rectangle.
+    void body(int shape)
     {
         const std::string ind = "        ";
-        o << "template <> __device__ __forceinline__ void " << kernel_name(block) << "_body<" << (border ? "true" : "false")
-          << ">(const KfArgs &a, const int ox, const int oy";
+        o << "__device__ __forceinline__ void " << kernel_name(block) << "_frame" << shape
+          << "(const KfArgs &a, const int ox, const int oy, const KfRect &rc";
         for (auto &g : groups)
             for (int k : g) o << ", " << (f32 ? "float" : "unsigned") << " *__restrict__ " << smem_name(k);
         o << ")\n{\n    const int W = a.W, H = a.H;\n    (void)H;\n";
@@ -218,31 +246,30 @@ struct Gen {
             for (int k : g) o << " " << k;
             o << " over the tile + halo (" << hx << "," << hy << ")\n";
             o << "    for (int i = threadIdx.x; i < " << rw * rh << "; i += blockDim.x) {\n";
-            o << "        const int y = oy - " << hy << " + i / " << rw << ", x = ox - " << hx << " + i % " << rw << ";\n";
-            if (border && !b.torus)
-                o << "        if (y < 0 || y >= H || x < 0 || x >= W || y < a.r0 - " << hy << " || y >= a.r1 + " << hy
-                  << ") continue;\n";
+            o << "        const int y = oy - " << hy << " + i / " << rw << ", x = ox - " << hx << " + i % " << rw
+              << ";\n";
+            if (!b.torus)
+                o << "        if (y < 0 || y >= H || x < 0 || x >= W || y < a.r0 - " << hy << " || y >= a.r1 + "
+                  << hy << ") continue;\n";
             std::map<int, std::string> memo;
             for (int k : g) {
-                std::string v = eval(p->n_inputs + k, memo, gs, border, ind);
+                std::string v = eval(p->n_inputs + k, memo, gs, ind);
                 o << ind << smem_name(k) << "[i] = " << (f32 ? v : "kf_pack(" + v + ")") << ";\n";
             }
             o << "    }\n    __syncthreads();\n";
         }
-        // sink
         o << "    for (int i = threadIdx.x; i < " << TW * TH << "; i += blockDim.x) {\n";
         o << "        const int y = oy + i / " << TW << ", x = ox + i % " << TW << ";\n";
-        o << "        if (y >= a.r1 || x >= W) continue;\n";
+        o << "        if (y >= rc.y1 || x >= rc.x1) continue;\n";
         std::map<int, std::string> memo;
-        std::string v = eval(p->n_inputs + b.sink, memo, {}, border, ind);
+        std::string v = eval(p->n_inputs + b.sink, memo, {}, ind);
         o << ind << (f32 ? "kf_stf" : "kf_sti") << "(a.out, a.out_base, W, y, x, " << v << ");\n";
         o << "    }\n}\n\n";
     }
 
-    std::string run()
+    void run()
     {
         for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
-        if (b.ext.size() > 16) fail(KF_ERR_ARG, "block reads more than 16 external images");
         // staged kernels grouped by (hx, hy), descending hx+hy (topological)
         std::map<std::pair<int, int>, std::vector<int>> byhalo;
         for (int k : b.staged) byhalo[{b.hx.at(k), b.hy.at(k)}].push_back(k);
@@ -252,52 +279,471 @@ struct Gen {
             return l.first + l.second > r.first + r.second;
         });
         for (auto &kk : keys) groups.push_back(byhalo[kk]);
-
-        o << "// generated by libkfuse codegen: block " << block << " kernels {";
-        for (int k : b.kernels) o << " " << k;
-        o << " } sink " << b.sink << (b.torus ? " (torus)" : "") << "\n";
-        o << "#include \"kf_device.cuh\"\n\n";
-        for (int k : b.kernels)
-            if (!p->ops[k].lut.empty()) {
-                o << "__device__ const int kf_lut_" << block << "_" << k << "[" << p->ops[k].lut.size() << "] = {";
-                for (size_t i = 0; i < p->ops[k].lut.size(); i++) o << (i ? "," : "") << p->ops[k].lut[i];
-                o << "};\n";
-            }
-        o << "template <bool BORDER> __device__ void " << kernel_name(block) << "_body(const KfArgs &a, int ox, int oy";
-        for (auto &g : groups)
-            for (size_t j = 0; j < g.size(); j++) o << ", " << (f32 ? "float" : "unsigned") << " *__restrict__";
-        o << ");\n";
-        body(false);
-        body(true);
         int smem = 0;
+        for (int shape = 0; shape < 2; shape++) {
+            TW = shape == 0 ? kFrameTiles[0][0] : kFrameTiles[1][0];
+            TH = shape == 0 ? kFrameTiles[0][1] : kFrameTiles[1][1];
+            body(shape);
+        }
         for (auto &g : groups)
-            for (int k : g) smem += RW(k) * RH(k) * 4;
+            for (int k : g) {
+                int n = 0;
+                for (int s = 0; s < 2; s++)
+                    n = std::max(n, (kFrameTiles[s][0] + 2 * b.hx.at(k)) * (kFrameTiles[s][1] + 2 * b.hy.at(k)));
+                smem += n * 4;
+            }
         if (smem > 48 * 1024) fail(KF_ERR_ARG, "fused block needs more than 48 KB of shared memory");
-        o << "extern \"C\" __global__ void __launch_bounds__(256) " << kernel_name(block)
-          << "(const __grid_constant__ KfArgs a)\n{\n";
+        // dispatcher for frame CTAs
+        o << "__device__ __forceinline__ void " << kernel_name(block) << "_frame(const KfArgs &a, int cta)\n{\n";
         for (auto &g : groups)
-            for (int k : g)
-                o << "    __shared__ " << (f32 ? "float " : "unsigned ") << smem_name(k) << "[" << RW(k) * RH(k)
-                  << "];\n";
-        o << "    const int ox = blockIdx.x * " << TW << ";\n";
-        o << "    const int oy = a.r0 + blockIdx.y * " << TH << ";\n";
-        o << "    const bool interior = ox >= " << b.Rx << " && ox + " << TW + b.Rx << " <= a.W && oy >= " << b.Ry
-          << " && oy + " << TH + b.Ry << " <= a.H && oy + " << TH << " <= a.r1;\n";
-        std::string args = "a, ox, oy";
+            for (int k : g) {
+                int n = 0;
+                for (int s = 0; s < 2; s++)
+                    n = std::max(n, (kFrameTiles[s][0] + 2 * b.hx.at(k)) * (kFrameTiles[s][1] + 2 * b.hy.at(k)));
+                o << "    __shared__ " << (f32 ? "float " : "unsigned ") << smem_name(k) << "[" << n << "];\n";
+            }
+        std::string sargs;
         for (auto &g : groups)
-            for (int k : g) args += ", " + smem_name(k);
-        o << "    if (interior) " << kernel_name(block) << "_body<false>(" << args << ");\n";
-        o << "    else " << kernel_name(block) << "_body<true>(" << args << ");\n}\n";
-        return o.str();
+            for (int k : g) sargs += ", " + smem_name(k);
+        o << "    int r = 0;\n";
+        o << "    while (r + 1 < a.n_rect && cta >= a.rect[r + 1].cta0) r++;\n";
+        o << "    const KfRect &rc = a.rect[r];\n";
+        o << "    const int t = cta - rc.cta0;\n";
+        o << "    if (rc.shape == 0) {\n";
+        o << "        " << kernel_name(block) << "_frame0(a, rc.x0 + (t % rc.ntx) * " << kFrameTiles[0][0]
+          << ", rc.y0 + (t / rc.ntx) * " << kFrameTiles[0][1] << ", rc" << sargs << ");\n";
+        o << "    } else {\n";
+        o << "        " << kernel_name(block) << "_frame1(a, rc.x0 + (t % rc.ntx) * " << kFrameTiles[1][0]
+          << ", rc.y0 + (t / rc.ntx) * " << kFrameTiles[1][1] << ", rc" << sargs << ");\n";
+        o << "    }\n}\n\n";
+    }
+};
+
+// ================================================================== interior
+// Fast path: one warp streams a column chunk down a strip of rows.
+//
+// Schedule.  Let HY(i) be the rows of image i the block needs
+// above/below the sink row (BlockInfo::hy for kernels, ext_hy for external
+// images) and L = max HY over the external images.  At iteration t the warp
+//   - has external image e at row  t - L + HY(e)  (prefetched D iterations ago),
+//   - computes kernel k at row     t - L + HY(k)  (as late as possible),
+// so the sink (HY = 0) emits row t - L.  A consumer k reads its producer i at
+// iteration offset HY(k) - HY(i) + dy <= 0: per-image register rings of P
+// slots indexed by iteration mod P; the loop body is emitted P times so every
+// ring index is a compile-time constant (no register moves).
+struct StreamGen {
+    const kf_pipeline *p;
+    const BlockInfo &b;
+    const StreamInfo &si;
+    int block;
+    bool f32;
+    std::ostringstream &o;
+    int tmp = 0;
+    ProgEmitter pe;
+    std::map<int, int> slot;   // external image -> slot
+    // per-iteration memo: (image, ring slot, column) -> unpacked value variable
+    std::map<std::tuple<int, int, int>, std::string> val_memo;
+    std::map<std::pair<std::string, int>, std::string> shfl_memo;   // (var, lane offset) -> shuffled var
+
+    StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
+        : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
+    {
+    }
+
+    static constexpr int V = kStreamV;
+    std::string KV() const { return f32 ? "float" : "I4"; }
+    std::string RT() const { return f32 ? "float" : "unsigned"; }   // ring storage type
+    std::string var() { return "v" + std::to_string(tmp++); }
+    int HY(int img) const { return si.hy.at(img); }
+    static int md(int a, int m) { return ((a % m) + m) % m; }
+    std::string ring(int img, int s, int v) const
+    {
+        return "r" + std::to_string(img) + "_" + std::to_string(s) + "_" + std::to_string(v);
+    }
+
+    // value of image img at ring slot s, column v of this lane (unpacked)
+    std::string value(int img, int s, int v, const std::string &ind)
+    {
+        auto key = std::make_tuple(img, s, v);
+        auto it = val_memo.find(key);
+        if (it != val_memo.end()) return it->second;
+        std::string r = ring(img, s, v);
+        if (!f32) {
+            std::string t = var();
+            o << ind << "const I4 " << t << " = kf_unpack(" << r << ");\n";
+            r = t;
+        }
+        val_memo[key] = r;
+        return r;
+    }
+
+    // value at column offset q (relative to this lane's first column) of a row
+    // whose V per-lane values are `row`: own register or a warp shuffle.
+    std::string at_col(const std::vector<std::string> &row, int q, const std::string &ind)
+    {
+        if (q >= 0 && q < V) return row[q];
+        int lo = q >= 0 ? q / V : -((-q + V - 1) / V);
+        int idx = q - lo * V;
+        auto key = std::make_pair(row[idx], lo);
+        auto it = shfl_memo.find(key);
+        if (it != shfl_memo.end()) return it->second;
+        std::string t = var();
+        o << ind << "const " << KV() << " " << t << " = " << (lo < 0 ? "kf_shup(" : "kf_shdn(") << row[idx] << ", "
+          << std::abs(lo) << ");\n";
+        shfl_memo[key] = t;
+        return t;
+    }
+
+    // acc = sum_i c_i * v_i over non-zero coefficients (emitted as FMA chain)
+    std::string lincomb(std::vector<std::pair<double, std::string>> terms, const std::string &ind)
+    {
+        // start from a unit-coefficient term when there is one (no multiply)
+        std::stable_partition(terms.begin(), terms.end(), [](const auto &t) { return t.first == 1.0; });
+        std::string acc;
+        for (auto &t : terms) {
+            if (t.first == 0.0) continue;
+            std::string c = f32 ? fconst(t.first) : iconst((long long)t.first);
+            std::string nv = var();
+            if (acc.empty()) {
+                if (t.first == 1.0)
+                    o << ind << "const " << KV() << " " << nv << " = " << t.second << ";\n";
+                else
+                    o << ind << "const " << KV() << " " << nv << " = kf_mul1(" << c << ", " << t.second << ");\n";
+            } else if (t.first == 1.0) {
+                o << ind << "const " << KV() << " " << nv << " = kf_add(" << acc << ", " << t.second << ");\n";
+            } else if (t.first == -1.0) {
+                o << ind << "const " << KV() << " " << nv << " = kf_sub(" << acc << ", " << t.second << ");\n";
+            } else {
+                o << ind << "const " << KV() << " " << nv << " = kf_mac(" << acc << ", " << c << ", " << t.second
+                  << ");\n";
+            }
+            acc = nv;
+        }
+        if (acc.empty()) {
+            acc = var();
+            o << ind << "const " << KV() << " " << acc << " = " << (f32 ? "0.0f" : "kf_i4(0)") << ";\n";
+        }
+        return acc;
+    }
+
+    // kernel k at iteration slot j: emits code, stores its V values into its
+    // ring slot j, and memoises the unpacked values.
+    void kernel(int k, int j, const std::string &ind)
+    {
+        const Op &op = p->ops[k];
+        const int img = p->n_inputs + k;
+        const int P = si.P;
+        std::vector<std::string> res(V);
+        if (op.kind == POINT) {
+            std::vector<std::vector<std::string>> ins;
+            for (int in : op.inputs) {
+                int s = md(j + HY(img) - HY(in), P);
+                std::vector<std::string> row;
+                for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
+                ins.push_back(row);
+            }
+            for (int v = 0; v < V; v++) {
+                std::vector<std::string> loads;
+                for (auto &r : ins) loads.push_back(r[v]);
+                res[v] = pe.emit(o, op, k, loads, ind);
+            }
+        } else {
+            const int in = op.inputs[0];
+            const int rx = op.mw / 2, ry = op.mh / 2;
+            auto rowvals = [&](int dy) {
+                int s = md(j + HY(img) - HY(in) + dy, P);
+                std::vector<std::string> row;
+                for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
+                return row;
+            };
+            std::vector<std::string> acc(V);
+            const Separable &sp = si.sep.at(k);
+            if (sp.ok) {
+                // vertical pass in the lane's own columns, then horizontal taps
+                std::vector<std::vector<std::string>> rows;
+                for (int dy = -ry; dy <= ry; dy++) rows.push_back(sp.col[dy + ry] != 0.0 ? rowvals(dy)
+                                                                                         : std::vector<std::string>());
+                std::vector<std::string> vs(V);
+                for (int v = 0; v < V; v++) {
+                    std::vector<std::pair<double, std::string>> terms;
+                    for (int dy = -ry; dy <= ry; dy++)
+                        if (sp.col[dy + ry] != 0.0) terms.push_back({sp.col[dy + ry], rows[dy + ry][v]});
+                    vs[v] = lincomb(terms, ind);
+                }
+                for (int v = 0; v < V; v++) {
+                    std::vector<std::pair<double, std::string>> terms;
+                    for (int dx = -rx; dx <= rx; dx++)
+                        if (sp.row[dx + rx] != 0.0) terms.push_back({sp.row[dx + rx], at_col(vs, v + dx, ind)});
+                    acc[v] = lincomb(terms, ind);
+                }
+            } else {
+                std::vector<std::vector<std::pair<double, std::string>>> terms(V);
+                for (int dy = -ry; dy <= ry; dy++) {
+                    bool any = false;
+                    for (int dx = -rx; dx <= rx; dx++) any |= op.mask[(size_t)(dy + ry) * op.mw + dx + rx] != 0.0;
+                    if (!any) continue;
+                    std::vector<std::string> row = rowvals(dy);
+                    for (int dx = -rx; dx <= rx; dx++) {
+                        double m = op.mask[(size_t)(dy + ry) * op.mw + dx + rx];
+                        if (m == 0.0) continue;
+                        for (int v = 0; v < V; v++) terms[v].push_back({m, at_col(row, v + dx, ind)});
+                    }
+                }
+                for (int v = 0; v < V; v++) acc[v] = lincomb(terms[v], ind);
+            }
+            for (int v = 0; v < V; v++)
+                res[v] = op.prog.empty() ? acc[v] : pe.emit(o, op, k, std::vector<std::string>{acc[v]}, ind);
+        }
+        for (int v = 0; v < V; v++) {
+            std::string r = res[v];
+            if (!f32) {   // narrowing at the kernel boundary
+                std::string t = var();
+                o << ind << "const I4 " << t << " = kf_satu8(" << r << ");\n";
+                r = t;
+                if (img != p->n_inputs + b.sink || si.depth.at(img) > 1)
+                    o << ind << ring(img, j, v) << " = kf_pack(" << r << ");\n";
+            } else {
+                o << ind << ring(img, j, v) << " = " << r << ";\n";
+            }
+            val_memo[std::make_tuple(img, j, v)] = r;
+        }
+    }
+
+    // prefetch of external image slot s for iteration (it) into ring slot rs
+    void load(int img, int rs, const std::string &it, const std::string &ind)
+    {
+        int s = slot.at(img);
+        std::string row = var();
+        o << ind << "const int " << row << " = min(max(ys - " << 2 * si.L - HY(img) << " + (" << it << "), a.base[" << s
+          << "]), a.rlast[" << s << "]);\n";
+        std::string ptr = "g" + std::to_string(s) + " + " + row + " * W";
+        if (si.vec) {
+            std::string q = var();
+            if (f32) {
+                o << ind << "const float4 " << q << " = kf_ld4f(" << ptr << ");\n";
+                const char *c[4] = {"x", "y", "z", "w"};
+                for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
+            } else {
+                o << ind << "const uint4 " << q << " = kf_ld4u(" << ptr << ");\n";
+                const char *c[4] = {"x", "y", "z", "w"};
+                for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
+            }
+        } else {
+            for (int v = 0; v < V; v++)
+                o << ind << ring(img, rs, v) << " = __ldg(" << ptr << " + cl" << v << ");\n";
+        }
+    }
+
+    void run()
+    {
+        for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
+        const int P = si.P, D = si.D, L = si.L, HL = si.HL;
+        const std::string ind = "        ";
+        o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast(const KfArgs &a, const int item)\n{\n";
+        o << "    const int lane = threadIdx.x & 31;\n";
+        o << "    const int W = a.W;\n";
+        o << "    const int chunk = item % a.n_chunks, strip = item / a.n_chunks;\n";
+        o << "    const int x = a.fx0 + (chunk * " << 32 - 2 * HL << " + lane - " << HL << ") * " << V << ";\n";
+        o << "    const bool xst = lane >= " << HL << " && lane < " << 32 - HL << " && x < a.fx1;\n";
+        o << "    const int ys = a.fy0 + strip * a.strip;\n";
+        o << "    const int ye = min(ys + a.strip, a.fy1);\n";
+        o << "    const int nit = ye - ys + " << 2 * L << ";\n";
+        if (si.vec) {
+            o << "    const int xl = min(max(x, 0), W - " << V << ");\n";
+        } else {
+            o << "    const int xl = 0;\n";
+            for (int v = 0; v < V; v++) o << "    const int cl" << v << " = min(max(x + " << v << ", 0), W - 1);\n";
+        }
+        for (int img : b.ext) {
+            int s = slot.at(img);
+            o << "    const " << RT() << " *__restrict__ g" << s << " = (const " << RT() << " *)a.img[" << s
+              << "] + xl - a.base[" << s << "] * W;\n";
+        }
+        // ring registers
+        std::set<int> imgs(b.ext.begin(), b.ext.end());
+        for (int k : b.kernels) imgs.insert(p->n_inputs + k);
+        for (int img : imgs) {
+            o << "    " << RT();
+            bool first = true;
+            for (int s = 0; s < P; s++)
+                for (int v = 0; v < V; v++) {
+                    o << (first ? " " : ", ") << ring(img, s, v) << " = 0";
+                    first = false;
+                }
+            o << ";\n";
+        }
+        // prologue: iterations 0 .. D-1
+        for (int it = 0; it < D; it++)
+            for (int img : b.ext) load(img, it % P, std::to_string(it), "    ");
+        std::string optr = "(" + RT() + " *)a.out + x - a.out_base * W";
+        o << "    " << RT() << " *__restrict__ gout = " << optr << ";\n";
+        o << "    for (int u = 0; u < nit; u += " << P << ") {\n";
+        for (int j = 0; j < P; j++) {
+            val_memo.clear();
+            shfl_memo.clear();
+            o << "      {   // iteration u + " << j << "\n";
+            for (int img : b.ext) load(img, (j + D) % P, "u + " + std::to_string(j + D), ind);
+            for (int k : b.kernels) kernel(k, j, ind);
+            // sink row = ys - 2L + iteration
+            const int simg = p->n_inputs + b.sink;
+            o << ind << "const int yo = ys - " << 2 * L << " + u + " << j << ";\n";
+            o << ind << "if (xst && yo >= ys && yo < ye) {\n";
+            if (!si.vec) {
+                for (int v = 0; v < V; v++) {
+                    std::string val = f32 ? ring(simg, j, v) : "kf_pack(" + val_memo[std::make_tuple(simg, j, v)] + ")";
+                    o << ind << "    if (x + " << v << " < a.fx1) gout[yo * W + " << v << "] = " << val << ";\n";
+                }
+            } else if (f32) {
+                o << ind << "    kf_st4f(gout + yo * W";
+                for (int v = 0; v < V; v++) o << ", " << ring(simg, j, v);
+                o << ");\n";
+            } else {
+                o << ind << "    kf_st4u(gout + yo * W";
+                for (int v = 0; v < V; v++) o << ", kf_pack(" << val_memo[std::make_tuple(simg, j, v)] << ")";
+                o << ");\n";
+            }
+            o << ind << "}\n";
+            o << "      }\n";
+        }
+        o << "    }\n}\n\n";
     }
 };
 
 }  // namespace
 
-std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block, int tile_w, int tile_h)
+// ------------------------------------------------------------ block analysis
+
+// Rank-1 factorisation m[j][i] = col[j] * row[i], exact in double.  Integer
+// masks (u8x4) get integer factors (primitive row vector), float masks that
+// are integers times a power of two get the same factors with the scale folded
+// into the row (e.g. Gaussian/16 = [1,2,1] (x) [1,2,1]/16, exact in float32).
+static Separable factor(const Op &op, bool integer)
 {
-    Gen g(p, b, block, tile_w > 0 ? tile_w : 32, tile_h > 0 ? tile_h : 8);
-    return g.run();
+    Separable s;
+    const int mw = op.mw, mh = op.mh;
+    double scale = 1.0;
+    bool ints = true;
+    for (double v : op.mask) ints &= std::floor(v) == v && std::fabs(v) < 1e9;
+    if (!ints && !integer) {
+        for (int e = 1; e <= 24 && !ints; e++) {
+            scale = std::ldexp(1.0, -e);
+            ints = true;
+            for (double v : op.mask) {
+                double w = v / scale;
+                ints &= std::floor(w) == w && std::fabs(w) < 1e9;
+            }
+        }
+        if (!ints) scale = 1.0;
+    }
+    if (!ints) return s;   // general float masks: direct 2-D taps (exact float order not needed, but keep simple)
+    std::vector<long long> A(op.mask.size());
+    for (size_t q = 0; q < A.size(); q++) A[q] = (long long)(op.mask[q] / scale);
+    int jr = -1;
+    for (int j = 0; j < mh && jr < 0; j++)
+        for (int i = 0; i < mw; i++)
+            if (A[(size_t)j * mw + i] != 0) { jr = j; break; }
+    if (jr < 0) return s;
+    long long g = 0;
+    for (int i = 0; i < mw; i++) g = std::gcd(g, std::llabs(A[(size_t)jr * mw + i]));
+    std::vector<long long> row(mw), col(mh);
+    int ip = -1;
+    for (int i = 0; i < mw; i++) {
+        row[i] = A[(size_t)jr * mw + i] / g;
+        if (row[i] != 0 && ip < 0) ip = i;
+    }
+    if (row[ip] < 0)
+        for (auto &r : row) r = -r;
+    for (int j = 0; j < mh; j++) {
+        long long a = A[(size_t)j * mw + ip];
+        if (a % row[ip] != 0) return s;
+        col[j] = a / row[ip];
+    }
+    for (int j = 0; j < mh; j++)
+        for (int i = 0; i < mw; i++)
+            if (col[j] * row[i] != A[(size_t)j * mw + i]) return s;
+    // sign: prefer the factor with more positive coefficients in the column
+    int neg = 0, pos = 0;
+    for (long long c : col) { neg += c < 0; pos += c > 0; }
+    if (neg > pos) {
+        for (auto &c : col) c = -c;
+        for (auto &r : row) r = -r;
+    }
+    s.ok = true;
+    for (int j = 0; j < mh; j++) s.col.push_back((double)col[j]);
+    for (int i = 0; i < mw; i++) s.row.push_back((double)row[i] * scale);
+    return s;
+}
+
+StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
+{
+    StreamInfo si;
+    si.vec = p->W % kStreamV == 0;
+    for (int img : b.ext) si.hy[img] = b.ext_hy.at(img);
+    for (int k : b.kernels) si.hy[p->n_inputs + k] = b.hy.at(k);
+    si.L = b.Ry;
+    si.HL = std::max(1, (b.Rx + kStreamV - 1) / kStreamV);
+    // history depth of every image, in iterations
+    int maxdepth_ext = 1, maxdepth = 1;
+    for (auto &kv : si.hy) si.depth[kv.first] = 1;
+    for (int k : b.kernels) {
+        const Op &op = p->ops[k];
+        const int img = p->n_inputs + k;
+        for (int in : op.inputs) {
+            int d = si.hy[in] - si.hy[img] + op.ry() + 1;
+            si.depth[in] = std::max(si.depth[in], d);
+        }
+        if (op.kind == LOCAL) si.sep[k] = factor(op, p->dtype != KF_F32);
+    }
+    for (auto &kv : si.depth) {
+        bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
+        (ext ? maxdepth_ext : maxdepth) = std::max(ext ? maxdepth_ext : maxdepth, kv.second);
+    }
+    // prefetch distance and ring period: P >= depth_ext + D, P >= every depth
+    si.D = 4;
+    si.P = std::max(maxdepth, maxdepth_ext + si.D);
+    // register estimate: live ring values (depth per image, D prefetched rows)
+    int live = 0;
+    for (auto &kv : si.depth) {
+        bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
+        live += (kv.second + (ext ? si.D : 0)) * kStreamV;
+    }
+    si.live_regs = live;
+    si.ok = b.Rx <= 2 * kStreamV * 4 && live <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
+    return si;
+}
+
+std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
+{
+    if (b.ext.size() > KF_MAX_IMG_HOST) fail(KF_ERR_ARG, "block reads more than 16 external images");
+    std::ostringstream o;
+    StreamInfo si = stream_info(p, b);
+    o << "// generated by libkfuse codegen: block " << block << " kernels {";
+    for (int k : b.kernels) o << " " << k;
+    o << " } sink " << b.sink << (b.torus ? " (torus)" : "") << "; interior path "
+      << (si.ok ? "streaming" : "none") << " (P=" << si.P << " D=" << si.D << " HL=" << si.HL << " L=" << si.L
+      << " live~" << si.live_regs << ")\n";
+    o << "#include \"kf_device.cuh\"\n\n";
+    for (int k : b.kernels)
+        if (!p->ops[k].lut.empty()) {
+            o << "__device__ const int kf_lut_" << block << "_" << k << "[" << p->ops[k].lut.size() << "] = {";
+            for (size_t i = 0; i < p->ops[k].lut.size(); i++) o << (i ? "," : "") << p->ops[k].lut[i];
+            o << "};\n";
+        }
+    FrameGen fg(p, b, block, o);
+    fg.run();
+    if (si.ok) {
+        StreamGen sg(p, b, si, block, o);
+        sg.run();
+    }
+    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << kMinCtasPerSm << ") " << kernel_name(block)
+      << "(const __grid_constant__ KfArgs a)\n{\n";
+    o << "    const int cta = blockIdx.x;\n";
+    o << "    if (cta < a.frame_ctas) { " << kernel_name(block) << "_frame(a, cta); return; }\n";
+    // one warp per CTA: the item index and the trip count are CTA-uniform, so
+    // the warp shuffles of the interior path need no convergence barriers
+    if (si.ok) o << "    " << kernel_name(block) << "_fast(a, cta - a.frame_ctas);\n";
+    o << "}\n";
+    return o.str();
 }
 
 }  // namespace kf

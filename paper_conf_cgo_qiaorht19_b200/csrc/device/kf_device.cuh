@@ -9,16 +9,34 @@
 #pragma once
 
 #define KF_MAX_IMG 16
+#define KF_MAX_RECT 4
 
+// A border-frame rectangle of the slow (index-exchange) path, tiled by one of
+// two tile shapes (0: 32 x 8 for the top/bottom frame, 1: 8 x 32 for the
+// left/right frame).  CTAs [cta0, cta0 + ntx * nty) of the launch cover it.
+struct KfRect {
+    int x0, x1, y0, y1;
+    int shape, ntx, nty, cta0;
+};
+
+// Launch arguments of one fused block kernel (__grid_constant__).  Mirrors the
+// geometry computed by runtime.cu.
 struct KfArgs {
     const void *img[KF_MAX_IMG];   // external images of the block (slot order)
     int base[KF_MAX_IMG];          // global row held by row 0 of each buffer
+    int rlast[KF_MAX_IMG];         // last global row held by each buffer
     void *out;                     // block output image
     int out_base;                  // global row held by row 0 of `out`
     int W, H;                      // image size (global)
     int r0, r1;                    // output rows computed by this launch
-    int tiles_x;                   // v1 tiling
-    int tiles_y;
+    // border frame: slow path, CTAs [0, frame_ctas)
+    KfRect rect[KF_MAX_RECT];
+    int n_rect, frame_ctas;
+    // interior: streaming fast path, one warp per item, CTAs [frame_ctas, ...)
+    int fx0, fx1, fy0, fy1;        // interior output rectangle (x multiple of 4)
+    int strip;                     // output rows per item
+    int n_chunks;                  // column chunks of (32 - 2*HL) * 4 columns
+    int n_items;                   // n_chunks * number of strips
 };
 
 // ------------------------------------------------------------ border map
@@ -146,3 +164,31 @@ __device__ __forceinline__ void kf_sti(void *p, int base, int W, int y, int x, I
 {
     ((unsigned *)p)[(size_t)(y - base) * W + x] = kf_pack(v);
 }
+
+// 128-bit accesses of the streaming path (4 pixels per lane)
+__device__ __forceinline__ float4 kf_ld4f(const float *p) { return __ldg((const float4 *)p); }
+__device__ __forceinline__ uint4 kf_ld4u(const unsigned *p) { return __ldg((const uint4 *)p); }
+__device__ __forceinline__ void kf_st4f(float *p, float a, float b, float c, float d)
+{
+    *(float4 *)p = make_float4(a, b, c, d);
+}
+__device__ __forceinline__ void kf_st4u(unsigned *p, unsigned a, unsigned b, unsigned c, unsigned d)
+{
+    *(uint4 *)p = make_uint4(a, b, c, d);
+}
+#define KF_FULL 0xffffffffu
+__device__ __forceinline__ float kf_shup(float v, int d) { return __shfl_up_sync(KF_FULL, v, d); }
+__device__ __forceinline__ float kf_shdn(float v, int d) { return __shfl_down_sync(KF_FULL, v, d); }
+__device__ __forceinline__ I4 kf_shup(I4 v, int d)
+{
+    return I4{__shfl_up_sync(KF_FULL, v.x, d), __shfl_up_sync(KF_FULL, v.y, d), __shfl_up_sync(KF_FULL, v.z, d),
+              __shfl_up_sync(KF_FULL, v.w, d)};
+}
+__device__ __forceinline__ I4 kf_shdn(I4 v, int d)
+{
+    return I4{__shfl_down_sync(KF_FULL, v.x, d), __shfl_down_sync(KF_FULL, v.y, d),
+              __shfl_down_sync(KF_FULL, v.z, d), __shfl_down_sync(KF_FULL, v.w, d)};
+}
+// first product of an accumulation (mask coefficient m)
+__device__ __forceinline__ float kf_mul1(float m, float v) { return m * v; }
+__device__ __forceinline__ I4 kf_mul1(int m, I4 v) { return I4{m * v.x, m * v.y, m * v.z, m * v.w}; }

@@ -120,13 +120,39 @@ bool header_legal(const kf_pipeline *p, const std::set<int> &P);
 BlockInfo analyse_block(const kf_pipeline *p, const std::vector<int> &kernels);
 
 // codegen.cpp
+constexpr int kStreamV = 4;                              // pixels per lane of the interior path
+constexpr int kThreads = 32;                             // threads per CTA (both paths): one warp
+constexpr int kMinCtasPerSm = 16;                        // __launch_bounds__ min blocks (<= 128 regs)
+constexpr int KF_MAX_IMG_HOST = 16;                      // = KF_MAX_IMG of kf_device.cuh
+constexpr int kFrameTiles[2][2] = {{32, 8}, {8, 32}};    // frame tile shapes (w, h)
+
+struct Separable {                // rank-1 mask: m[j][i] = col[j] * row[i]
+    bool ok = false;
+    std::vector<double> col, row;
+};
+
+// Interior streaming schedule of one block (codegen.cpp StreamGen)
+struct StreamInfo {
+    bool ok = false;              // the block has an interior fast path
+    bool vec = false;             // W % 4 == 0: 128-bit loads/stores
+    int L = 0;                    // rows of lag of the sink behind the newest input row
+    int HL = 1;                   // halo lanes per warp side
+    int P = 1;                    // ring period = loop body copies
+    int D = 4;                    // prefetch distance (iterations)
+    int live_regs = 0;            // estimate of ring registers
+    std::map<int, int> hy;        // image -> rows needed around the sink row
+    std::map<int, int> depth;     // image -> history depth (iterations)
+    std::map<int, Separable> sep; // local kernel -> factorisation
+};
+
 std::string kernel_name(int block);
-std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block, int tile_w, int tile_h);
+StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b);
+std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block);
 
 // runtime.cu
 void prepare(kf_pipeline *p, kf_plan *plan);
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
-         void *stream, int row0, int row1, int in_row0);
+         void *stream, int row0, int row1, int in_row0, int in_row1);
 void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
               void *stream);
 void release_plan(kf_plan *plan);

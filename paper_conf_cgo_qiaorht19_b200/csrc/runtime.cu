@@ -19,6 +19,7 @@
 #include <sstream>
 
 #include "kf_internal.h"
+#include "device/kf_device.cuh"
 
 namespace kf {
 
@@ -41,6 +42,7 @@ struct Driver {
     CUresult (*launchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
                              CUstream, void **, void **) = nullptr;
     CUresult (*getErrorString)(CUresult, const char **) = nullptr;
+    CUresult (*occupancy)(int *, CUfunction, int, size_t) = nullptr;
 };
 
 static Driver &driver()
@@ -67,6 +69,7 @@ static Driver &driver()
         get("cuModuleUnload", (void **)&d.moduleUnload);
         get("cuLaunchKernel", (void **)&d.launchKernel);
         get("cuGetErrorString", (void **)&d.getErrorString);
+        get("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void **)&d.occupancy);
     });
     if (!err.empty() || !d.launchKernel) fail(KF_ERR_CUDA, "CUDA unavailable:" + err);
     return d;
@@ -152,7 +155,9 @@ static std::string compile_cubin(const std::string &src, const std::string &name
 struct CompiledBlock {
     CUmodule mod = nullptr;
     CUfunction fn = nullptr;
-    int tile_w = 32, tile_h = 8, threads = 256;
+    StreamInfo si;               // interior schedule the kernel was generated with
+    int ctas_per_sm = 1;         // occupancy of the kernel (cuOccupancy...)
+    int num_sms = 148;
     std::string source;
     ~CompiledBlock()
     {
@@ -175,7 +180,7 @@ struct Runtime {
 // Compile-only path usable without a GPU (build() warms the in-tree cache).
 std::string compile_block_cubin(const kf_pipeline *p, const kf_plan *plan, int i)
 {
-    return compile_cubin(generate_block(p, plan->info[i], i, 0, 0), kernel_name(i));
+    return compile_cubin(generate_block(p, plan->info[i], i), kernel_name(i));
 }
 
 void prepare(kf_pipeline *p, kf_plan *plan)
@@ -189,7 +194,7 @@ void prepare(kf_pipeline *p, kf_plan *plan)
     p->rt->device = dev;
     plan->compiled.clear();
     for (size_t i = 0; i < plan->blocks.size(); i++) {
-        std::string src = generate_block(p, plan->info[i], (int)i, 0, 0);
+        std::string src = generate_block(p, plan->info[i], (int)i);
         uint64_t h = fnv1a(src);
         auto it = p->rt->modules.find(h);
         if (it == p->rt->modules.end()) {
@@ -198,6 +203,10 @@ void prepare(kf_pipeline *p, kf_plan *plan)
             cu_check(d.moduleLoadData(&cb->mod, cubin.data()), "cuModuleLoadData");
             cu_check(d.moduleGetFunction(&cb->fn, cb->mod, kernel_name((int)i).c_str()), "cuModuleGetFunction");
             cb->source = src;
+            cb->si = stream_info(p, plan->info[i]);
+            cu_check(d.occupancy(&cb->ctas_per_sm, cb->fn, kThreads, 0), "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+            cb->ctas_per_sm = std::max(1, cb->ctas_per_sm);
+            KF_CUDA(cudaDeviceGetAttribute(&cb->num_sms, cudaDevAttrMultiProcessorCount, dev));
             it = p->rt->modules.emplace(h, cb).first;
         }
         plan->compiled.push_back(it->second);
@@ -224,8 +233,76 @@ void prepare(kf_pipeline *p, kf_plan *plan)
 // Executes rows [row0, row1) of every output.  Full-image run: row0 = 0,
 // row1 = H, inputs hold all rows (in_row0 = 0).  Band run: inputs hold rows
 // from in_row0; each block computes its sink over the rows its consumers need.
+// Launch geometry of one block: the interior rectangle whose
+// whole input footprint is inside the image goes to the streaming path (one
+// warp per (column chunk, row strip) item, strip height chosen so the items
+// fill whole waves of resident warps); the rest of rows [r0, r1) -- the border
+// frame -- is tiled by the index-exchange path.  Returns the grid size.
+static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlock &cb)
+{
+    const int W = a.W, H = a.H, V = kStreamV;
+    const StreamInfo &si = cb.si;
+    int fx0 = 0, fx1 = 0, fy0 = 0, fy1 = 0;
+    bool fast = si.ok;
+    if (fast) {
+        fy0 = std::max(a.r0, b.Ry);
+        fy1 = std::min(a.r1, H - b.Ry);
+        if (si.vec) {
+            fx0 = (b.Rx + V - 1) / V * V;
+            fx1 = (W - b.Rx) / V * V;
+        } else {
+            fx0 = b.Rx;
+            fx1 = W - b.Rx;
+        }
+        fast = fx1 > fx0 && fy1 > fy0;
+    }
+    struct R { int x0, x1, y0, y1, shape; };
+    std::vector<R> rects;
+    if (fast) {
+        rects = {{0, W, a.r0, fy0, 0}, {0, W, fy1, a.r1, 0}, {0, fx0, fy0, fy1, 1}, {fx1, W, fy0, fy1, 1}};
+    } else {
+        rects = {{0, W, a.r0, a.r1, 0}};
+    }
+    int cta = 0;
+    a.n_rect = 0;
+    for (const R &r : rects) {
+        if (r.x1 <= r.x0 || r.y1 <= r.y0) continue;
+        KfRect &k = a.rect[a.n_rect++];
+        k.x0 = r.x0; k.x1 = r.x1; k.y0 = r.y0; k.y1 = r.y1; k.shape = r.shape;
+        k.ntx = (r.x1 - r.x0 + kFrameTiles[r.shape][0] - 1) / kFrameTiles[r.shape][0];
+        k.nty = (r.y1 - r.y0 + kFrameTiles[r.shape][1] - 1) / kFrameTiles[r.shape][1];
+        k.cta0 = cta;
+        cta += k.ntx * k.nty;
+    }
+    a.frame_ctas = cta;
+    if (!fast) return (unsigned)cta;
+    a.fx0 = fx0; a.fx1 = fx1; a.fy0 = fy0; a.fy1 = fy1;
+    const int chunk_w = (32 - 2 * si.HL) * V;
+    a.n_chunks = (fx1 - fx0 + chunk_w - 1) / chunk_w;
+    const int Hf = fy1 - fy0;
+    const int warps_per_cta = 1;
+    const long long slots = (long long)cb.num_sms * cb.ctas_per_sm;   // resident CTAs per wave
+    // strip height: minimise waves x rows streamed per item (iterations rounded to P)
+    long long best = -1;
+    int best_strip = Hf;
+    for (int ns = 1; ns <= Hf; ns++) {
+        const int S = (Hf + ns - 1) / ns;
+        if (ns > 1 && (Hf + S - 1) / S != ns) continue;          // same S as a smaller ns
+        const long long items = (long long)a.n_chunks * ((Hf + S - 1) / S);
+        const long long ctas = (items + warps_per_cta - 1) / warps_per_cta;
+        const long long waves = (ctas + slots - 1) / slots;
+        const long long iters = (S + 2 * si.L + si.P - 1) / si.P * si.P;
+        const long long cost = waves * iters;
+        if (best < 0 || cost < best) { best = cost; best_strip = S; }
+        if (items > 64 * slots * warps_per_cta) break;
+    }
+    a.strip = best_strip;
+    a.n_items = a.n_chunks * ((Hf + best_strip - 1) / best_strip);
+    return (unsigned)(cta + (a.n_items + warps_per_cta - 1) / warps_per_cta);
+}
+
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
-         void *stream, int row0, int row1, int in_row0)
+         void *stream, int row0, int row1, int in_row0, int in_row1)
 {
     if (n_in != p->n_inputs || (n_in && !din)) fail(KF_ERR_ARG, "wrong number of inputs");
     if (n_out != (int)p->outputs.size() || (n_out && !dout)) fail(KF_ERR_ARG, "wrong number of outputs");
@@ -254,8 +331,12 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
     }
     // where each image lives
     std::vector<void *> ptr(nimg, nullptr);
-    std::vector<int> base(nimg, 0);
-    for (int i = 0; i < p->n_inputs; i++) { ptr[i] = const_cast<void *>(din[i]); base[i] = in_row0; }
+    std::vector<int> base(nimg, 0), rlast(nimg, p->H - 1);
+    for (int i = 0; i < p->n_inputs; i++) {
+        ptr[i] = const_cast<void *>(din[i]);
+        base[i] = in_row0;
+        rlast[i] = band ? in_row1 - 1 : p->H - 1;
+    }
     for (auto &kv : plan->workspace) { ptr[kv.first] = kv.second; base[kv.first] = 0; }
     std::vector<std::pair<int, int>> band_copies;   // (image, output slot) copied at the end
     for (int j = 0; j < n_out; j++) {
@@ -271,17 +352,13 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
     for (size_t bi = 0; bi < plan->blocks.size(); bi++) {
         const BlockInfo &b = plan->info[bi];
         const CompiledBlock &cb = *plan->compiled[bi];
-        struct Args {
-            const void *img[16];
-            int base[16];
-            void *out;
-            int out_base;
-            int W, H, r0, r1, tiles_x, tiles_y;
-        } a;
+        KfArgs a;
         std::memset(&a, 0, sizeof a);
         for (size_t s = 0; s < b.ext.size(); s++) {
-            a.img[s] = ptr[b.ext[s]];
-            a.base[s] = base[b.ext[s]];
+            const int e = b.ext[s];
+            a.img[s] = ptr[e];
+            a.base[s] = base[e];
+            a.rlast[s] = rlast[e];
         }
         int sink = p->n_inputs + b.sink;
         a.out = ptr[sink];
@@ -290,13 +367,10 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         a.H = p->H;
         a.r0 = blo[bi];
         a.r1 = bhi[bi];
-        a.tiles_x = (p->W + cb.tile_w - 1) / cb.tile_w;
-        a.tiles_y = (a.r1 - a.r0 + cb.tile_h - 1) / cb.tile_h;
-        if (a.tiles_y <= 0) continue;
-        if (a.tiles_y > 65535) fail(KF_ERR_ARG, "image too tall for the v1 grid");
+        if (a.r1 <= a.r0) continue;
+        unsigned grid = launch_geometry(a, b, cb);
         void *params[] = {&a};
-        cu_check(d.launchKernel(cb.fn, a.tiles_x, a.tiles_y, 1, cb.threads, 1, 1, 0, st, params, nullptr),
-                 "cuLaunchKernel");
+        cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
     }
     for (auto &c : band_copies) {
         const char *src = (const char *)plan->workspace[c.first] + (size_t)row0 * p->W * 4;
@@ -326,7 +400,7 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     cudaStream_t s = (cudaStream_t)stream;
     for (int i = 0; i < n_in; i++) KF_CUDA(cudaMemcpyAsync(rt.stage_in[i], hin[i], bytes, cudaMemcpyHostToDevice, s));
     std::vector<const void *> din(rt.stage_in.begin(), rt.stage_in.end());
-    run(p, plan, din.data(), n_in, rt.stage_out.data(), n_out, stream, 0, p->H, 0);
+    run(p, plan, din.data(), n_in, rt.stage_out.data(), n_out, stream, 0, p->H, 0, p->H);
     for (int j = 0; j < n_out; j++) KF_CUDA(cudaMemcpyAsync(hout[j], rt.stage_out[j], bytes, cudaMemcpyDeviceToHost, s));
     KF_CUDA(cudaStreamSynchronize(s));
 }
