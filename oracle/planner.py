@@ -16,6 +16,11 @@ Contents, each in the paper's notation:
   brute_force()   exact maximum of Eq. 1 over all partitions into legal blocks
                   (the paper's "exhaustive search")
 
+Parity unpinned (R-4, R-7): the local-to-local locality gain of Eq. 3
+(garbled, read as IS*tg/ts) and the B200 profile's STAGED recompute factor have
+no numeric example in the paper; only the point-based / point-to-local weights
+(328/256/eps) and the Eq. 9 sizes are pinned.
+
 Weights are lexicographic pairs (real, eps-count) with the real part in fixed
 point q = floor(w * 2^20 + 0.5) (reading O1-i): sums are exact, so ties
 ("the first one encountered") are decided identically here
