@@ -167,25 +167,29 @@ def config_dict(cfg_name, spec, plan, extra=None) -> dict:
 # --------------------------------------------------------------------- GPU
 
 
-def time_plan(plan, ins, outs, steps, warmup, stream, torch, launches):
-    """Times exactly `steps` kf_run calls; returns (ms/step total, mean per-step
-    event time of the plan's kernels)."""
+def time_plan(plan, ins, outs, steps, warmup, stream, torch):
+    """Times exactly `steps` kf_run calls (one step = one whole plan over one
+    image, rotating over the buffer sets).  The steps are captured once into a
+    CUDA graph so that the host-side launch cost of the ctypes binding is out of
+    the timed region; the graph replay is bracketed by CUDA events on the
+    launching stream.  Returns ms per step."""
     n = len(ins)
     with torch.cuda.stream(stream):
         for i in range(warmup):
             plan.run([ins[i % n]], [outs[i % n]], stream)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
-    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=stream):
+        for i in range(steps):
+            plan.run([ins[i % n]], [outs[i % n]], stream)
+    g.replay()                                       # warm replay (untimed)
+    torch.cuda.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     t0.record(stream)
-    for i in range(steps):
-        ev[i][0].record(stream)
-        plan.run([ins[i % n]], [outs[i % n]], stream)
-        ev[i][1].record(stream)
+    g.replay()
     t1.record(stream)
     torch.cuda.synchronize()
-    per = [a.elapsed_time(b) for a, b in ev]
-    return t0.elapsed_time(t1) / steps, sum(per) / len(per)
+    return t0.elapsed_time(t1) / steps
 
 
 def bench_single(args, cfg_name, spec, seed) -> None:
@@ -219,21 +223,21 @@ def bench_single(args, cfg_name, spec, seed) -> None:
         p, plan = plans[kind]
         if kind == args.plan:
             with ClockSampler(dev) as cs:
-                ms, kern_ms = time_plan(plan, ins, outs, args.steps, args.warmup, stream, torch, plan.num_launches)
+                ms = time_plan(plan, ins, outs, args.steps, args.warmup, stream, torch)
             clocks = cs.summary()
         else:
-            ms, kern_ms = time_plan(plan, ins, outs, max(20, args.steps // 4), args.warmup, stream, torch,
-                                    plan.num_launches)
+            ms = time_plan(plan, ins, outs, max(50, args.steps // 4), args.warmup, stream, torch)
         ab = ALG_BYTES.get(spec["name"], {}).get(kind)
         results[kind] = {"ms_per_step": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
                          "launches": plan.num_launches, "alg_bytes_per_px": ab,
-                         "alg_gbs": round(ab * px / (ms * 1e-3) / 1e9, 1) if ab else None,
-                         "kernel_ms": round(kern_ms, 5)}
+                         "alg_gbs": round(ab * px / (ms * 1e-3) / 1e9, 1) if ab else None}
     head = results[args.plan]
     peaks = load_peaks()
     _, hplan = plans[args.plan]
     ab = head["alg_bytes_per_px"] or 8
-    achieved = ab * px / (head["kernel_ms"] * 1e-3) / 1e9
+    # the headline plan is one launch per step, so the step time of the graph
+    # replay is that kernel's average launch duration
+    achieved = ab * px / (head["ms_per_step"] * 1e-3) / 1e9
     traffic = ncu_traffic(cfg_name, args.plan)
     roofline = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
@@ -343,7 +347,7 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="kfuse", choices=["kfuse", "reference"])
     ap.add_argument("--config", default="C3")

@@ -27,6 +27,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <functional>
 #include <numeric>
 #include <sstream>
@@ -320,17 +321,29 @@ struct FrameGen {
 };
 
 // ================================================================== interior
-// Fast path: one warp streams a column chunk down a strip of rows.
+// Streaming path: one warp streams a column chunk along a strip of rows.
 //
 // Schedule.  Let HY(i) be the rows of image i the block needs
 // above/below the sink row (BlockInfo::hy for kernels, ext_hy for external
-// images) and L = max HY over the external images.  At iteration t the warp
+// images) and L = max HY over the external images.  Rows are counted in the
+// strip's streaming direction (dir = +1 downward, -1 upward: r' = r or
+// H-1-r).  At iteration t the warp
 //   - has external image e at row  t - L + HY(e)  (prefetched D iterations ago),
 //   - computes kernel k at row     t - L + HY(k)  (as late as possible),
 // so the sink (HY = 0) emits row t - L.  A consumer k reads its producer i at
-// iteration offset HY(k) - HY(i) + dy <= 0: per-image register rings of P
+// iteration offset HY(k) - HY(i) + dy' <= 0: per-image register rings of P
 // slots indexed by iteration mod P; the loop body is emitted P times so every
 // ring index is a compile-time constant (no register moves).
+//
+// Image edges (index exchange, R-12): a consumer reads its
+// producer at B(p) with ITS OWN border mode.
+//   - vertical: the strip that starts at an image edge (top strip downward,
+//     bottom strip upward) peels its first Q iterations, in which every tap row
+//     r' + dy' < 0 is redirected statically to the ring slot of row B(r' + dy')
+//     (always an already computed row) or to the constant;
+//   - horizontal: in the first/last column chunk the lane holding columns
+//     0..3 (W-4..W-1) replaces the taps that would come from the neighbour
+//     lane by its own register at B(c) (or the constant): one select per tap.
 struct StreamGen {
     const kf_pipeline *p;
     const BlockInfo &b;
@@ -343,7 +356,10 @@ struct StreamGen {
     std::map<int, int> slot;   // external image -> slot
     // per-iteration memo: (image, ring slot, column) -> unpacked value variable
     std::map<std::tuple<int, int, int>, std::string> val_memo;
-    std::map<std::pair<std::string, int>, std::string> shfl_memo;   // (var, lane offset) -> shuffled var
+    std::map<std::tuple<std::string, int, int>, std::string> shfl_memo;   // (var, lane offset, edge key)
+    // variant being emitted
+    int dir = 1;
+    bool el = false, er = false;
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
@@ -356,9 +372,28 @@ struct StreamGen {
     std::string var() { return "v" + std::to_string(tmp++); }
     int HY(int img) const { return si.hy.at(img); }
     static int md(int a, int m) { return ((a % m) + m) % m; }
+    bool is_ext(int img) const { return std::binary_search(b.ext.begin(), b.ext.end(), img); }
+    // Ring slot of image img at iteration offset `off` (<= 0: past rows; +D:
+    // the prefetch of an external image) seen from loop-body copy j.  Unrolled:
+    // slot = iteration mod P.  Rolled (one body copy, rings shifted by register
+    // moves at the end of every iteration): slot = age (+D for external images).
+    int sl(int img, int off, int j) const
+    {
+        if (!si.rolled) return md(j + off, si.P);
+        return -off + (is_ext(img) ? si.D : 0);
+    }
+    int ring_len(int img) const
+    {
+        if (!si.rolled) return si.P;
+        return si.depth.at(img) + (is_ext(img) ? si.D : 0);
+    }
     std::string ring(int img, int s, int v) const
     {
         return "r" + std::to_string(img) + "_" + std::to_string(s) + "_" + std::to_string(v);
+    }
+    std::string cval(const Op &op) const
+    {
+        return f32 ? fconst(op.constant) : "kf_i4(" + iconst((int)op.constant) + ")";
     }
 
     // value of image img at ring slot s, column v of this lane (unpacked)
@@ -377,19 +412,50 @@ struct StreamGen {
         return r;
     }
 
+    // Border map of one axis at an edge of an image of (large) size n, for the
+    // columns/rows just outside: returns the in-image index relative to the
+    // edge (0 = the edge pixel), or -1 for the constant.  c < 0 = outside.
+    static int edge_map(int mode, int c)
+    {
+        switch (mode) {
+        case KF_CLAMP: return 0;
+        case KF_MIRROR: return -c - 1;
+        case KF_MIRROR101: return -c;
+        default: return -1;   // KF_CONSTANT
+        }
+    }
+
     // value at column offset q (relative to this lane's first column) of a row
-    // whose V per-lane values are `row`: own register or a warp shuffle.
-    std::string at_col(const std::vector<std::string> &row, int q, const std::string &ind)
+    // whose V per-lane values are `row`: own register or a warp shuffle; in an
+    // edge chunk the edge lane substitutes the border-mapped own register.
+    std::string at_col(const std::vector<std::string> &row, int q, const Op &op, const std::string &csub,
+                       const std::string &ind)
     {
         if (q >= 0 && q < V) return row[q];
         int lo = q >= 0 ? q / V : -((-q + V - 1) / V);
         int idx = q - lo * V;
-        auto key = std::make_pair(row[idx], lo);
+        const bool edge = (q < 0 && el) || (q >= V && er);
+        const int ekey = edge ? op.mode * 64 + q : -1000;
+        auto key = std::make_tuple(row[idx], lo, ekey);
         auto it = shfl_memo.find(key);
         if (it != shfl_memo.end()) return it->second;
         std::string t = var();
         o << ind << "const " << KV() << " " << t << " = " << (lo < 0 ? "kf_shup(" : "kf_shdn(") << row[idx] << ", "
           << std::abs(lo) << ");\n";
+        if (edge) {
+            std::string sub;
+            if (q < 0) {
+                int m = edge_map(op.mode, q);   // column q < 0 of the lane at x = 0
+                sub = m < 0 ? csub : row[m];
+            } else {
+                int m = edge_map(op.mode, -(q - V) - 1);   // column W + (q - V) of the lane at x = W - V
+                sub = m < 0 ? csub : row[V - 1 - m];
+            }
+            std::string t2 = var();
+            o << ind << "const " << KV() << " " << t2 << " = (" << (q < 0 ? "x == 0" : "x == W - 4") << ") ? "
+              << sub << " : " << t << ";\n";
+            t = t2;
+        }
         shfl_memo[key] = t;
         return t;
     }
@@ -426,18 +492,45 @@ struct StreamGen {
         return acc;
     }
 
+    // Row of producer `in` needed by consumer k (image kimg) at primed tap
+    // offset dyp, in iteration slot j.  `u` >= 0: the iteration index is the
+    // compile-time constant u of a peeled edge iteration (rows relative to the
+    // strip start = the image edge), so taps outside the image are remapped;
+    // u < 0: steady state, no remap.  Returns an empty vector for a constant row.
+    std::vector<std::string> tap_row(int kimg, const Op &op, int in, int dyp, int j, int u, bool &is_const,
+                                     const std::string &ind)
+    {
+        const int L = si.L;
+        int s = sl(in, HY(kimg) - HY(in) + dyp, j);
+        is_const = false;
+        if (u >= 0) {
+            const int rk = u - 2 * L + HY(kimg);   // consumer row (primed, 0 = edge row)
+            const int rr = rk + dyp;
+            if (rr < 0 && rk >= 0) {
+                const int m = edge_map(op.mode, rr);
+                if (m < 0) {
+                    is_const = true;
+                    return {};
+                }
+                s = sl(in, m + 2 * L - HY(in) - u, j);   // the iteration that computed row m of `in`
+            }
+        }
+        std::vector<std::string> row;
+        for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
+        return row;
+    }
+
     // kernel k at iteration slot j: emits code, stores its V values into its
     // ring slot j, and memoises the unpacked values.
-    void kernel(int k, int j, const std::string &ind)
+    void kernel(int k, int j, int u, const std::string &ind)
     {
         const Op &op = p->ops[k];
         const int img = p->n_inputs + k;
-        const int P = si.P;
         std::vector<std::string> res(V);
         if (op.kind == POINT) {
             std::vector<std::vector<std::string>> ins;
             for (int in : op.inputs) {
-                int s = md(j + HY(img) - HY(in), P);
+                int s = sl(in, HY(img) - HY(in), j);
                 std::vector<std::string> row;
                 for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
                 ins.push_back(row);
@@ -450,43 +543,69 @@ struct StreamGen {
         } else {
             const int in = op.inputs[0];
             const int rx = op.mw / 2, ry = op.mh / 2;
-            auto rowvals = [&](int dy) {
-                int s = md(j + HY(img) - HY(in) + dy, P);
-                std::vector<std::string> row;
-                for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
-                return row;
-            };
+            // mask row of primed tap offset dyp (upward strips flip the mask)
+            auto mrow = [&](int dyp) { return ry + dir * dyp; };
             std::vector<std::string> acc(V);
             const Separable &sp = si.sep.at(k);
             if (sp.ok) {
                 // vertical pass in the lane's own columns, then horizontal taps
-                std::vector<std::vector<std::string>> rows;
-                for (int dy = -ry; dy <= ry; dy++) rows.push_back(sp.col[dy + ry] != 0.0 ? rowvals(dy)
-                                                                                         : std::vector<std::string>());
+                std::vector<std::pair<double, std::vector<std::string>>> rows;
+                std::vector<double> cterms;   // coefficients of constant (exterior) rows
+                for (int dy = -ry; dy <= ry; dy++) {   // mask-row order in both directions (same rounding)
+                    const int dyp = dir * dy;
+                    const double c = sp.col[mrow(dyp)];
+                    if (c == 0.0) continue;
+                    bool isc = false;
+                    auto r = tap_row(img, op, in, dyp, j, u, isc, ind);
+                    if (isc) cterms.push_back(c);
+                    else rows.push_back({c, r});
+                }
                 std::vector<std::string> vs(V);
+                std::string cst;
+                if (!cterms.empty()) {
+                    double cs = 0.0;
+                    for (double c : cterms) cs += c;
+                    cst = var();
+                    o << ind << "const " << KV() << " " << cst << " = kf_mul1(" << (f32 ? fconst(cs) : iconst((long long)cs))
+                      << ", " << cval(op) << ");\n";
+                }
                 for (int v = 0; v < V; v++) {
                     std::vector<std::pair<double, std::string>> terms;
-                    for (int dy = -ry; dy <= ry; dy++)
-                        if (sp.col[dy + ry] != 0.0) terms.push_back({sp.col[dy + ry], rows[dy + ry][v]});
+                    for (auto &r : rows) terms.push_back({r.first, r.second[v]});
+                    if (!cst.empty()) terms.push_back({1.0, cst});
                     vs[v] = lincomb(terms, ind);
+                }
+                // an exterior column of a CONSTANT consumer is c in every row: c * sum(col)
+                std::string csub;
+                if (op.mode == KF_CONSTANT && (el || er)) {
+                    double cs = 0.0;
+                    for (double c : sp.col) cs += c;
+                    csub = var();
+                    o << ind << "const " << KV() << " " << csub << " = kf_mul1("
+                      << (f32 ? fconst(cs) : iconst((long long)cs)) << ", " << cval(op) << ");\n";
                 }
                 for (int v = 0; v < V; v++) {
                     std::vector<std::pair<double, std::string>> terms;
                     for (int dx = -rx; dx <= rx; dx++)
-                        if (sp.row[dx + rx] != 0.0) terms.push_back({sp.row[dx + rx], at_col(vs, v + dx, ind)});
+                        if (sp.row[dx + rx] != 0.0)
+                            terms.push_back({sp.row[dx + rx], at_col(vs, v + dx, op, csub, ind)});
                     acc[v] = lincomb(terms, ind);
                 }
             } else {
                 std::vector<std::vector<std::pair<double, std::string>>> terms(V);
                 for (int dy = -ry; dy <= ry; dy++) {
+                    const int dyp = dir * dy;
+                    const int mr = mrow(dyp);
                     bool any = false;
-                    for (int dx = -rx; dx <= rx; dx++) any |= op.mask[(size_t)(dy + ry) * op.mw + dx + rx] != 0.0;
+                    for (int dx = -rx; dx <= rx; dx++) any |= op.mask[(size_t)mr * op.mw + dx + rx] != 0.0;
                     if (!any) continue;
-                    std::vector<std::string> row = rowvals(dy);
+                    bool isc = false;
+                    std::vector<std::string> row = tap_row(img, op, in, dyp, j, u, isc, ind);
                     for (int dx = -rx; dx <= rx; dx++) {
-                        double m = op.mask[(size_t)(dy + ry) * op.mw + dx + rx];
+                        double m = op.mask[(size_t)mr * op.mw + dx + rx];
                         if (m == 0.0) continue;
-                        for (int v = 0; v < V; v++) terms[v].push_back({m, at_col(row, v + dx, ind)});
+                        for (int v = 0; v < V; v++)
+                            terms[v].push_back({m, isc ? cval(op) : at_col(row, v + dx, op, cval(op), ind)});
                     }
                 }
                 for (int v = 0; v < V; v++) acc[v] = lincomb(terms[v], ind);
@@ -494,6 +613,7 @@ struct StreamGen {
             for (int v = 0; v < V; v++)
                 res[v] = op.prog.empty() ? acc[v] : pe.emit(o, op, k, std::vector<std::string>{acc[v]}, ind);
         }
+        const int ws = sl(img, 0, j);
         for (int v = 0; v < V; v++) {
             std::string r = res[v];
             if (!f32) {   // narrowing at the kernel boundary
@@ -501,52 +621,100 @@ struct StreamGen {
                 o << ind << "const I4 " << t << " = kf_satu8(" << r << ");\n";
                 r = t;
                 if (img != p->n_inputs + b.sink || si.depth.at(img) > 1)
-                    o << ind << ring(img, j, v) << " = kf_pack(" << r << ");\n";
+                    o << ind << ring(img, ws, v) << " = kf_pack(" << r << ");\n";
             } else {
-                o << ind << ring(img, j, v) << " = " << r << ";\n";
+                o << ind << ring(img, ws, v) << " = " << r << ";\n";
             }
-            val_memo[std::make_tuple(img, j, v)] = r;
+            val_memo[std::make_tuple(img, ws, v)] = r;
         }
     }
 
-    // prefetch of external image slot s for iteration (it) into ring slot rs
+    // prefetch of external image `img` for iteration `it` into ring slot rs
     void load(int img, int rs, const std::string &it, const std::string &ind)
     {
         int s = slot.at(img);
+        std::string rp = "(ys - " + std::to_string(2 * si.L - HY(img)) + " + (" + it + "))";   // primed row
         std::string row = var();
-        o << ind << "const int " << row << " = min(max(ys - " << 2 * si.L - HY(img) << " + (" << it << "), a.base[" << s
-          << "]), a.rlast[" << s << "]);\n";
+        o << ind << "const int " << row << " = min(max(" << (dir > 0 ? rp : "(H - 1 - " + rp + ")") << ", a.base["
+          << s << "]), a.rlast[" << s << "]);\n";
         std::string ptr = "g" + std::to_string(s) + " + " + row + " * W";
+        const char *c[4] = {"x", "y", "z", "w"};
         if (si.vec) {
             std::string q = var();
-            if (f32) {
-                o << ind << "const float4 " << q << " = kf_ld4f(" << ptr << ");\n";
-                const char *c[4] = {"x", "y", "z", "w"};
-                for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
-            } else {
-                o << ind << "const uint4 " << q << " = kf_ld4u(" << ptr << ");\n";
-                const char *c[4] = {"x", "y", "z", "w"};
-                for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
-            }
+            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = " << (f32 ? "kf_ld4f(" : "kf_ld4u(")
+              << ptr << ");\n";
+            for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
         } else {
             for (int v = 0; v < V; v++)
                 o << ind << ring(img, rs, v) << " = __ldg(" << ptr << " + cl" << v << ");\n";
         }
     }
 
-    void run()
+    // One iteration (slot j).  u >= 0: peeled edge iteration with index u.
+    void iteration(int j, int u, const std::string &uexpr, const std::string &ind)
     {
-        for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
+        const int P = si.P, D = si.D, L = si.L;
+        val_memo.clear();
+        shfl_memo.clear();
+        o << ind.substr(2) << "{   // iteration " << uexpr << " + " << j << "\n";
+        for (int img : b.ext) load(img, sl(img, D, j), uexpr + " + " + std::to_string(j + D), ind);
+        for (int k : b.kernels) kernel(k, j, u, ind);
+        const int simg = p->n_inputs + b.sink;
+        const int ss = sl(simg, 0, j);
+        o << ind << "const int yp = ys - " << 2 * L << " + " << uexpr << " + " << j << ";\n";
+        o << ind << "if (xst && yp >= ys && yp < ye) {\n";
+        o << ind << "    const int yo = " << (dir > 0 ? "yp" : "H - 1 - yp") << ";\n";
+        if (!si.vec) {
+            for (int v = 0; v < V; v++) {
+                std::string val = f32 ? ring(simg, ss, v) : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
+                o << ind << "    if (x + " << v << " < a.fx1) gout[yo * W + " << v << "] = " << val << ";\n";
+            }
+        } else if (f32) {
+            o << ind << "    kf_st4f(gout + yo * W";
+            for (int v = 0; v < V; v++) o << ", " << ring(simg, ss, v);
+            o << ");\n";
+        } else {
+            o << ind << "    kf_st4u(gout + yo * W";
+            for (int v = 0; v < V; v++) o << ", kf_pack(" << val_memo[std::make_tuple(simg, ss, v)] << ")";
+            o << ");\n";
+        }
+        o << ind << "}\n";
+        if (si.rolled) {   // age every ring by one row
+            std::set<int> imgs(b.ext.begin(), b.ext.end());
+            for (int k : b.kernels) imgs.insert(p->n_inputs + k);
+            for (int img : imgs)
+                for (int a = ring_len(img) - 1; a >= 1; a--)
+                    for (int v = 0; v < V; v++) o << ind << ring(img, a, v) << " = " << ring(img, a - 1, v) << ";\n";
+        }
+        o << ind.substr(2) << "}\n";
+    }
+
+    static std::string vname(int dir, bool ve, bool l, bool r)
+    {
+        return std::string("_") + (dir > 0 ? "d" : "u") + (ve ? "e" : "i") + (l ? "L" : "") + (r ? "R" : "");
+    }
+
+    // One variant: direction, vertical edge at the strip start, left/right edge chunk.
+    void variant(int dir_, bool ve, bool l, bool r)
+    {
+        dir = dir_;
+        el = l;
+        er = r;
         const int P = si.P, D = si.D, L = si.L, HL = si.HL;
-        const std::string ind = "        ";
-        o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast(const KfArgs &a, const int item)\n{\n";
+        o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast" << vname(dir, ve, l, r)
+          << "(const KfArgs &a, const int chunk, const int strip)\n{\n";
         o << "    const int lane = threadIdx.x & 31;\n";
-        o << "    const int W = a.W;\n";
-        o << "    const int chunk = item % a.n_chunks, strip = item / a.n_chunks;\n";
+        o << "    const int W = a.W, H = a.H;\n    (void)H;\n";
         o << "    const int x = a.fx0 + (chunk * " << 32 - 2 * HL << " + lane - " << HL << ") * " << V << ";\n";
         o << "    const bool xst = lane >= " << HL << " && lane < " << 32 - HL << " && x < a.fx1;\n";
-        o << "    const int ys = a.fy0 + strip * a.strip;\n";
-        o << "    const int ye = min(ys + a.strip, a.fy1);\n";
+        // strip bounds in primed (streaming-direction) rows
+        o << "    const int ys0 = a.fy0 + strip * a.strip;\n";
+        o << "    const int ye0 = strip == a.n_strips - 1 ? a.fy1 : ys0 + a.strip;   // the last strip takes the rest\n";
+        if (dir > 0) {
+            o << "    const int ys = ys0, ye = ye0;\n";
+        } else {
+            o << "    const int ys = H - ye0, ye = H - ys0;\n";
+        }
         o << "    const int nit = ye - ys + " << 2 * L << ";\n";
         if (si.vec) {
             o << "    const int xl = min(max(x, 0), W - " << V << ");\n";
@@ -559,53 +727,71 @@ struct StreamGen {
             o << "    const " << RT() << " *__restrict__ g" << s << " = (const " << RT() << " *)a.img[" << s
               << "] + xl - a.base[" << s << "] * W;\n";
         }
-        // ring registers
         std::set<int> imgs(b.ext.begin(), b.ext.end());
         for (int k : b.kernels) imgs.insert(p->n_inputs + k);
         for (int img : imgs) {
             o << "    " << RT();
             bool first = true;
-            for (int s = 0; s < P; s++)
+            for (int s = 0; s < ring_len(img); s++)
                 for (int v = 0; v < V; v++) {
                     o << (first ? " " : ", ") << ring(img, s, v) << " = 0";
                     first = false;
                 }
             o << ";\n";
         }
-        // prologue: iterations 0 .. D-1
         for (int it = 0; it < D; it++)
-            for (int img : b.ext) load(img, it % P, std::to_string(it), "    ");
-        std::string optr = "(" + RT() + " *)a.out + x - a.out_base * W";
-        o << "    " << RT() << " *__restrict__ gout = " << optr << ";\n";
-        o << "    for (int u = 0; u < nit; u += " << P << ") {\n";
-        for (int j = 0; j < P; j++) {
-            val_memo.clear();
-            shfl_memo.clear();
-            o << "      {   // iteration u + " << j << "\n";
-            for (int img : b.ext) load(img, (j + D) % P, "u + " + std::to_string(j + D), ind);
-            for (int k : b.kernels) kernel(k, j, ind);
-            // sink row = ys - 2L + iteration
-            const int simg = p->n_inputs + b.sink;
-            o << ind << "const int yo = ys - " << 2 * L << " + u + " << j << ";\n";
-            o << ind << "if (xst && yo >= ys && yo < ye) {\n";
-            if (!si.vec) {
-                for (int v = 0; v < V; v++) {
-                    std::string val = f32 ? ring(simg, j, v) : "kf_pack(" + val_memo[std::make_tuple(simg, j, v)] + ")";
-                    o << ind << "    if (x + " << v << " < a.fx1) gout[yo * W + " << v << "] = " << val << ";\n";
-                }
-            } else if (f32) {
-                o << ind << "    kf_st4f(gout + yo * W";
-                for (int v = 0; v < V; v++) o << ", " << ring(simg, j, v);
-                o << ");\n";
-            } else {
-                o << ind << "    kf_st4u(gout + yo * W";
-                for (int v = 0; v < V; v++) o << ", kf_pack(" << val_memo[std::make_tuple(simg, j, v)] << ")";
-                o << ");\n";
-            }
-            o << ind << "}\n";
-            o << "      }\n";
+            for (int img : b.ext) load(img, si.rolled ? D - it : it % P, std::to_string(it), "    ");
+        o << "    " << RT() << " *__restrict__ gout = (" << RT() << " *)a.out + x - a.out_base * W;\n";
+        int u0 = 0;
+        if (ve) {
+            // peeled iterations in which some tap row lies beyond the edge
+            int need = 0;
+            for (int k : b.kernels)
+                if (p->ops[k].kind == LOCAL)
+                    need = std::max(need, 2 * L - HY(p->n_inputs + k) + p->ops[k].ry());
+            const int Q = (need + P - 1) / P * P;
+            for (int u = 0; u < Q; u++) iteration(u % P, u, std::to_string(u - u % P), "      ");
+            u0 = Q;
+        }
+        if (si.rolled) {
+            o << "    #pragma unroll 1\n";
+            o << "    for (int u = " << u0 << "; u < nit; u++) {\n";
+            iteration(0, -1, "u", "        ");
+        } else {
+            o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
+            for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
         }
         o << "    }\n}\n\n";
+    }
+
+    void run()
+    {
+        for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
+        // Variants (the variant is CTA-uniform):
+        //   interior strip, interior chunk   -- the hot loop, no border logic
+        //   interior strip, edge chunk       -- + lane selects at x == 0 / x == W-4
+        //   top edge strip (downward)        -- + peeled remapped prologue, selects
+        //   bottom edge strip (upward)       -- same in flipped row order
+        const bool hsel = si.edge_l || si.edge_r;
+        variant(1, false, false, false);
+        if (hsel) variant(1, false, si.edge_l, si.edge_r);
+        if (si.edge_v) {
+            variant(1, true, si.edge_l, si.edge_r);
+            variant(-1, true, si.edge_l, si.edge_r);
+        }
+        o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast(const KfArgs &a, const int item)\n{\n";
+        o << "    const int chunk = item % a.n_chunks, strip = item / a.n_chunks;\n";
+        if (si.edge_v) {
+            o << "    if (a.edge_t && strip == 0) { " << kernel_name(block) << "_fast" << vname(1, true, si.edge_l, si.edge_r)
+              << "(a, chunk, strip); return; }\n";
+            o << "    if (a.edge_b && strip == a.n_strips - 1) { " << kernel_name(block) << "_fast"
+              << vname(-1, true, si.edge_l, si.edge_r) << "(a, chunk, strip); return; }\n";
+        }
+        if (hsel)
+            o << "    if ((a.edge_l && chunk == 0) || (a.edge_r && chunk == a.n_chunks - 1)) { " << kernel_name(block)
+              << "_fast" << vname(1, false, si.edge_l, si.edge_r) << "(a, chunk, strip); return; }\n";
+        o << "    " << kernel_name(block) << "_fast" << vname(1, false, false, false) << "(a, chunk, strip);\n";
+        o << "}\n\n";
     }
 };
 
@@ -674,6 +860,15 @@ static Separable factor(const Op &op, bool integer)
     return s;
 }
 
+// Tuning knobs (diagnostics / sweeps): integer env var in [lo, hi] or the default.
+int env_int(const char *name, int dflt, int lo, int hi)
+{
+    const char *e = std::getenv(name);
+    if (!e || !*e) return dflt;
+    int v = std::atoi(e);
+    return std::min(hi, std::max(lo, v));
+}
+
 StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
 {
     StreamInfo si;
@@ -699,7 +894,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         (ext ? maxdepth_ext : maxdepth) = std::max(ext ? maxdepth_ext : maxdepth, kv.second);
     }
     // prefetch distance and ring period: P >= depth_ext + D, P >= every depth
-    si.D = 4;
+    si.D = env_int("KFUSE_PREFETCH", 4, 1, 16);
     si.P = std::max(maxdepth, maxdepth_ext + si.D);
     // register estimate: live ring values (depth per image, D prefetched rows)
     int live = 0;
@@ -708,6 +903,43 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         live += (kv.second + (ext ? si.D : 0)) * kStreamV;
     }
     si.live_regs = live;
+    // code size: scalar operations of one iteration (one body copy)
+    const int ch = p->dtype == KF_F32 ? 1 : 4;
+    long long ops = 0;
+    for (int k : b.kernels) {
+        const Op &op = p->ops[k];
+        if (op.kind == LOCAL) {
+            int nnz = 0;
+            for (double m : op.mask) nnz += m != 0.0;
+            const Separable &sp = si.sep.at(k);
+            int taps = sp.ok ? (int)(std::count_if(sp.col.begin(), sp.col.end(), [](double c) { return c != 0.0; }) +
+                                     std::count_if(sp.row.begin(), sp.row.end(), [](double c) { return c != 0.0; }))
+                             : nnz;
+            ops += (long long)(taps + 2 * op.rx() + (int)op.prog.size()) * kStreamV * ch;
+        } else {
+            ops += (long long)op.prog.size() * kStreamV * ch;
+        }
+    }
+    si.iter_ops = ops;
+    // image edges inside the streaming path: not for REPEAT
+    // (wrap reads the opposite side), horizontal only when every exterior tap of
+    // the edge lane maps into its own 4 pixels
+    bool rep = b.torus, hfit = true;
+    for (int k : b.kernels) {
+        const Op &op = p->ops[k];
+        if (op.kind != LOCAL) continue;
+        rep |= op.mode == KF_REPEAT;
+        hfit &= op.rx() <= (op.mode == KF_MIRROR101 ? kStreamV - 1 : kStreamV);
+    }
+    si.edge_v = !rep && p->H >= 4 * si.L + 2 * si.P + 8;
+    // unrolled: ~P copies per variant (4 variants + 2 peeled prologues); too
+    // much straight-line code for NVRTC/ptxas -> rolled body, vertical edges
+    // left to the frame path
+    const long long budget = env_int("KFUSE_CODE_BUDGET", 12000, 0, 1 << 30);
+    si.rolled = ops * si.P * 6 > budget;
+    if (si.rolled) si.edge_v = false;
+    si.edge_l = !rep && hfit && p->W >= 4 * kStreamV;
+    si.edge_r = si.edge_l && si.vec;
     si.ok = b.Rx <= 2 * kStreamV * 4 && live <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
     return si;
 }
@@ -721,7 +953,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     for (int k : b.kernels) o << " " << k;
     o << " } sink " << b.sink << (b.torus ? " (torus)" : "") << "; interior path "
       << (si.ok ? "streaming" : "none") << " (P=" << si.P << " D=" << si.D << " HL=" << si.HL << " L=" << si.L
-      << " live~" << si.live_regs << ")\n";
+      << " live~" << si.live_regs << " ops~" << si.iter_ops << (si.rolled ? " rolled" : " unrolled") << ")\n";
     o << "#include \"kf_device.cuh\"\n\n";
     for (int k : b.kernels)
         if (!p->ops[k].lut.empty()) {
@@ -735,7 +967,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
         StreamGen sg(p, b, si, block, o);
         sg.run();
     }
-    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << kMinCtasPerSm << ") " << kernel_name(block)
+    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << env_int("KFUSE_MINCTAS", kMinCtasPerSm, 1, 32) << ") " << kernel_name(block)
       << "(const __grid_constant__ KfArgs a)\n{\n";
     o << "    const int cta = blockIdx.x;\n";
     o << "    if (cta < a.frame_ctas) { " << kernel_name(block) << "_frame(a, cta); return; }\n";

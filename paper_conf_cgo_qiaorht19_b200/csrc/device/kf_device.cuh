@@ -36,7 +36,9 @@ struct KfArgs {
     int fx0, fx1, fy0, fy1;        // interior output rectangle (x multiple of 4)
     int strip;                     // output rows per item
     int n_chunks;                  // column chunks of (32 - 2*HL) * 4 columns
-    int n_items;                   // n_chunks * number of strips
+    int n_strips;                  // row strips (the last one takes the remainder)
+    int n_items;                   // n_chunks * n_strips
+    int edge_l, edge_r, edge_t, edge_b;   // image edges handled by the edge chunks / strips
 };
 
 // ------------------------------------------------------------ border map

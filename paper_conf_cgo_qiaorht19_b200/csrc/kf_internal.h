@@ -140,12 +140,17 @@ struct StreamInfo {
     int P = 1;                    // ring period = loop body copies
     int D = 4;                    // prefetch distance (iterations)
     int live_regs = 0;            // estimate of ring registers
+    bool rolled = false;          // one loop-body copy + ring shifts (big blocks)
+    long long iter_ops = 0;       // scalar operations per iteration (code-size estimate)
+    bool edge_v = false;          // top/bottom image edges handled by edge strips
+    bool edge_l = false, edge_r = false;   // left/right image edges handled by edge chunks
     std::map<int, int> hy;        // image -> rows needed around the sink row
     std::map<int, int> depth;     // image -> history depth (iterations)
     std::map<int, Separable> sep; // local kernel -> factorisation
 };
 
 std::string kernel_name(int block);
+int env_int(const char *name, int dflt, int lo, int hi);
 StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b);
 std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block);
 

@@ -233,28 +233,28 @@ void prepare(kf_pipeline *p, kf_plan *plan)
 // Executes rows [row0, row1) of every output.  Full-image run: row0 = 0,
 // row1 = H, inputs hold all rows (in_row0 = 0).  Band run: inputs hold rows
 // from in_row0; each block computes its sink over the rows its consumers need.
-// Launch geometry of one block: the interior rectangle whose
-// whole input footprint is inside the image goes to the streaming path (one
-// warp per (column chunk, row strip) item, strip height chosen so the items
-// fill whole waves of resident warps); the rest of rows [r0, r1) -- the border
-// frame -- is tiled by the index-exchange path.  Returns the grid size.
+// Launch geometry of one block.  The streaming path covers
+// the rectangle [fx0, fx1) x [fy0, fy1): the whole rows [r0, r1) when the
+// block's image edges can be handled by edge strips/chunks (index exchange
+// inside the streaming path), otherwise only the pixels whose whole input
+// footprint is inside the image.  Whatever remains -- the border frame -- is
+// tiled by the shared-memory index-exchange path.  One warp (= one CTA) per
+// (column chunk, row strip) item; the strip height is chosen so the items fill
+// whole waves of resident warps.  Returns the grid size.
 static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlock &cb)
 {
     const int W = a.W, H = a.H, V = kStreamV;
     const StreamInfo &si = cb.si;
     int fx0 = 0, fx1 = 0, fy0 = 0, fy1 = 0;
-    bool fast = si.ok;
+    bool fast = si.ok, top = false, bot = false;
     if (fast) {
-        fy0 = std::max(a.r0, b.Ry);
-        fy1 = std::min(a.r1, H - b.Ry);
-        if (si.vec) {
-            fx0 = (b.Rx + V - 1) / V * V;
-            fx1 = (W - b.Rx) / V * V;
-        } else {
-            fx0 = b.Rx;
-            fx1 = W - b.Rx;
-        }
-        fast = fx1 > fx0 && fy1 > fy0;
+        top = si.edge_v && a.r0 == 0;
+        bot = si.edge_v && a.r1 == H;
+        fy0 = top ? 0 : std::max(a.r0, b.Ry);
+        fy1 = bot ? H : std::min(a.r1, H - b.Ry);
+        fx0 = si.edge_l ? 0 : (si.vec ? (b.Rx + V - 1) / V * V : b.Rx);
+        fx1 = si.edge_r ? W : (si.vec ? (W - b.Rx) / V * V : W - b.Rx);
+        fast = fx1 > fx0 && fy1 - fy0 >= (top && bot ? 2 * std::max(1, si.L) : 1);
     }
     struct R { int x0, x1, y0, y1, shape; };
     std::vector<R> rects;
@@ -277,28 +277,35 @@ static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlo
     a.frame_ctas = cta;
     if (!fast) return (unsigned)cta;
     a.fx0 = fx0; a.fx1 = fx1; a.fy0 = fy0; a.fy1 = fy1;
+    a.edge_l = si.edge_l; a.edge_r = si.edge_r; a.edge_t = top; a.edge_b = bot;
     const int chunk_w = (32 - 2 * si.HL) * V;
     a.n_chunks = (fx1 - fx0 + chunk_w - 1) / chunk_w;
     const int Hf = fy1 - fy0;
-    const int warps_per_cta = 1;
-    const long long slots = (long long)cb.num_sms * cb.ctas_per_sm;   // resident CTAs per wave
-    // strip height: minimise waves x rows streamed per item (iterations rounded to P)
+    const long long slots = (long long)cb.num_sms * cb.ctas_per_sm;   // resident single-warp CTAs per wave
+    // n_strips = floor(Hf / S): strips of S rows, the last one takes the rest
+    // (< 2S).  Edge strips must be at least L rows so that no interior strip
+    // reads beyond the image; a top and a bottom edge need two strips.
+    const int min_strips = top && bot ? 2 : 1;
+    const int smin = top || bot ? std::max(1, si.L) : 1;
     long long best = -1;
-    int best_strip = Hf;
-    for (int ns = 1; ns <= Hf; ns++) {
-        const int S = (Hf + ns - 1) / ns;
-        if (ns > 1 && (Hf + S - 1) / S != ns) continue;          // same S as a smaller ns
-        const long long items = (long long)a.n_chunks * ((Hf + S - 1) / S);
-        const long long ctas = (items + warps_per_cta - 1) / warps_per_cta;
-        const long long waves = (ctas + slots - 1) / slots;
-        const long long iters = (S + 2 * si.L + si.P - 1) / si.P * si.P;
-        const long long cost = waves * iters;
-        if (best < 0 || cost < best) { best = cost; best_strip = S; }
-        if (items > 64 * slots * warps_per_cta) break;
+    int best_S = Hf / min_strips;
+    for (int ns = min_strips; ns <= std::max(min_strips, Hf / smin); ns++) {
+        const int S = Hf / ns;
+        if (ns > min_strips && Hf / (ns - 1) == S) continue;
+        const int nst = Hf / S;
+        const int last = Hf - (nst - 1) * S;
+        const long long items = (long long)a.n_chunks * nst;
+        const long long waves = (items + slots - 1) / slots;
+        auto iters = [&](int rows) { return (long long)(rows + 2 * si.L + si.P - 1) / si.P * si.P; };
+        // the wave containing the long last strip bounds the time
+        const long long cost = (waves - 1) * iters(S) + iters(last);
+        if (best < 0 || cost < best) { best = cost; best_S = S; }
+        if (items > 64 * slots) break;
     }
-    a.strip = best_strip;
-    a.n_items = a.n_chunks * ((Hf + best_strip - 1) / best_strip);
-    return (unsigned)(cta + (a.n_items + warps_per_cta - 1) / warps_per_cta);
+    a.strip = best_S;
+    a.n_strips = Hf / best_S;
+    a.n_items = a.n_chunks * a.n_strips;
+    return (unsigned)(cta + a.n_items);
 }
 
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
@@ -369,6 +376,10 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         a.r1 = bhi[bi];
         if (a.r1 <= a.r0) continue;
         unsigned grid = launch_geometry(a, b, cb);
+        if (const char *skip = getenv("KFUSE_DIAG_SKIP")) {   // timing diagnostics only: wrong results
+            if (!strcmp(skip, "frame")) { grid -= a.frame_ctas; a.frame_ctas = 0; a.n_rect = 0; }
+            if (!strcmp(skip, "fast")) { grid = a.frame_ctas; }
+        }
         void *params[] = {&a};
         cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
     }
