@@ -182,12 +182,13 @@ def time_plan(plan, ins, outs, steps, warmup, stream, torch):
     with torch.cuda.graph(g, stream=stream):
         for i in range(steps):
             plan.run([ins[i % n]], [outs[i % n]], stream)
-    g.replay()                                       # warm replay (untimed)
-    torch.cuda.synchronize()
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    t0.record(stream)
-    g.replay()
-    t1.record(stream)
+    with torch.cuda.stream(stream):                  # replay() launches on the current stream
+        g.replay()                                   # warm replay (untimed)
+        torch.cuda.synchronize()
+        t0.record(stream)
+        g.replay()
+        t1.record(stream)
     torch.cuda.synchronize()
     return t0.elapsed_time(t1) / steps
 

@@ -114,6 +114,79 @@ struct ProgEmitter {
         }
         return st.back();
     }
+
+    // Packed f32x2 form of a float program (two adjacent pixels per value).
+    // The postfix program is rebuilt as a tree (each value is consumed once)
+    // so that a MUL feeding an ADD/SUB becomes one FFMA2 -- the contraction
+    // nvcc performs on scalar code but not across the _rn pair intrinsics.
+    struct Node {
+        int op, arg;
+        double imm;
+        std::vector<int> ch;
+    };
+    std::string emit2(std::ostringstream &o, const Op &op, const std::vector<std::string> &loads,
+                      const std::string &ind)
+    {
+        std::vector<Node> nodes;
+        std::vector<int> st;
+        for (const Instr &in : op.prog) {
+            Node n{in.op, in.arg, in.imm, {}};
+            int arity = 0;
+            switch (in.op) {
+            case KF_OP_LOAD: case KF_OP_CONST: arity = 0; break;
+            case KF_OP_ABS: case KF_OP_NEG: case KF_OP_SQRT: case KF_OP_EXP: case KF_OP_LOG: arity = 1; break;
+            case KF_OP_CLAMP: arity = 3; break;
+            case KF_OP_SELECT_GT: arity = 4; break;
+            case KF_OP_SHR: case KF_OP_SHL: case KF_OP_SAT_U8: case KF_OP_LUT:
+                fail(KF_ERR_PROGRAM, "codegen: integer opcode in a float program");
+            default: arity = 2;
+            }
+            n.ch.assign(st.end() - arity, st.end());
+            st.resize(st.size() - arity);
+            nodes.push_back(n);
+            st.push_back((int)nodes.size() - 1);
+        }
+        std::function<std::string(int)> ev = [&](int i) -> std::string {
+            const Node &n = nodes[i];
+            auto is = [&](int c, int opc) { return nodes[c].op == opc; };
+            auto cst = [&](int c) { return fconst(nodes[c].imm); };
+            std::string e;
+            if (n.op == KF_OP_LOAD) return loads[op.kind == LOCAL ? 0 : n.arg];
+            if (n.op == KF_OP_CONST) return "kf2(" + fconst(n.imm) + ")";
+            if (n.op == KF_OP_ADD || n.op == KF_OP_SUB) {
+                const int a = n.ch[0], b = n.ch[1];
+                const bool add = n.op == KF_OP_ADD;
+                if (is(b, KF_OP_MUL)) {
+                    std::string x = ev(a), m0 = ev(nodes[b].ch[0]), m1 = ev(nodes[b].ch[1]);
+                    e = std::string(add ? "kf2_fma(" : "kf2_nfma(") + m0 + ", " + m1 + ", " + x + ")";
+                } else if (is(a, KF_OP_MUL)) {
+                    std::string m0 = ev(nodes[a].ch[0]), m1 = ev(nodes[a].ch[1]), y = ev(b);
+                    e = std::string(add ? "kf2_fma(" : "kf2_fms(") + m0 + ", " + m1 + ", " + y + ")";
+                } else {
+                    e = std::string(add ? "kf2_add(" : "kf2_sub(") + ev(a) + ", " + ev(b) + ")";
+                }
+            } else if (n.op == KF_OP_MUL && is(n.ch[1], KF_OP_CONST)) {
+                e = "kf2_mul1(" + cst(n.ch[1]) + ", " + ev(n.ch[0]) + ")";
+            } else if (n.op == KF_OP_MUL && is(n.ch[0], KF_OP_CONST)) {
+                e = "kf2_mul1(" + cst(n.ch[0]) + ", " + ev(n.ch[1]) + ")";
+            } else {
+                static const std::map<int, const char *> fn = {
+                    {KF_OP_MUL, "kf2_mul"}, {KF_OP_DIV, "kf2_div"}, {KF_OP_MIN, "kf2_min"}, {KF_OP_MAX, "kf2_max"},
+                    {KF_OP_POW, "kf2_pow"}, {KF_OP_ABS, "kf2_abs"}, {KF_OP_NEG, "kf2_neg"}, {KF_OP_SQRT, "kf2_sqrt"},
+                    {KF_OP_EXP, "kf2_exp"}, {KF_OP_LOG, "kf2_log"}, {KF_OP_CLAMP, "kf2_clamp"},
+                    {KF_OP_SELECT_GT, "kf2_sel_gt"}};
+                auto it = fn.find(n.op);
+                if (it == fn.end()) fail(KF_ERR_PROGRAM, "codegen: bad opcode");
+                e = std::string(it->second) + "(";
+                for (size_t c = 0; c < n.ch.size(); c++) e += (c ? ", " : "") + ev(n.ch[c]);
+                e += ")";
+            }
+            std::string t = var();
+            o << ind << "const F2 " << t << " = " << e << ";\n";
+            return t;
+        };
+        return ev(st.back());
+    }
 };
 
 // ====================================================================== frame
@@ -360,6 +433,7 @@ struct StreamGen {
     // variant being emitted
     int dir = 1;
     bool el = false, er = false;
+    bool pm = false;   // f32 values kept as packed pixel pairs (F2) for column-local math
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
@@ -371,6 +445,8 @@ struct StreamGen {
     std::string RT() const { return f32 ? "float" : "unsigned"; }   // ring storage type
     std::string var() { return "v" + std::to_string(tmp++); }
     int HY(int img) const { return si.hy.at(img); }
+    int NR() const { return pm ? V / 2 : V; }                         // ring registers per row
+    std::string RDT() const { return pm ? "F2" : RT(); }               // ring register type
     static int md(int a, int m) { return ((a % m) + m) % m; }
     bool is_ext(int img) const { return std::binary_search(b.ext.begin(), b.ext.end(), img); }
     // Ring slot of image img at iteration offset `off` (<= 0: past rows; +D:
@@ -380,12 +456,12 @@ struct StreamGen {
     int sl(int img, int off, int j) const
     {
         if (!si.rolled) return md(j + off, si.P);
-        return -off + (is_ext(img) ? si.D : 0);
+        return -off + (is_ext(img) && !si.sring ? si.D : 0);
     }
     int ring_len(int img) const
     {
         if (!si.rolled) return si.P;
-        return si.depth.at(img) + (is_ext(img) ? si.D : 0);
+        return si.depth.at(img) + (is_ext(img) && !si.sring ? si.D : 0);
     }
     std::string ring(int img, int s, int v) const
     {
@@ -397,8 +473,10 @@ struct StreamGen {
     }
 
     // value of image img at ring slot s, column v of this lane (unpacked)
+    std::string pval(int img, int s, int q) const { return ring(img, s, q); }
     std::string value(int img, int s, int v, const std::string &ind)
     {
+        if (pm) return ring(img, s, v / 2) + (v % 2 ? ".y" : ".x");
         auto key = std::make_tuple(img, s, v);
         auto it = val_memo.find(key);
         if (it != val_memo.end()) return it->second;
@@ -492,6 +570,32 @@ struct StreamGen {
         return acc;
     }
 
+    // packed form of lincomb over pixel pairs
+    std::string lincomb2(std::vector<std::pair<double, std::string>> terms, const std::string &ind)
+    {
+        std::stable_partition(terms.begin(), terms.end(), [](const auto &t) { return t.first == 1.0; });
+        std::string acc;
+        for (auto &t : terms) {
+            if (t.first == 0.0) continue;
+            std::string c = fconst(t.first), nv = var();
+            if (acc.empty())
+                o << ind << "const F2 " << nv << " = " << (t.first == 1.0 ? t.second : "kf2_mul1(" + c + ", " + t.second + ")")
+                  << ";\n";
+            else if (t.first == 1.0)
+                o << ind << "const F2 " << nv << " = kf2_add(" << acc << ", " << t.second << ");\n";
+            else if (t.first == -1.0)
+                o << ind << "const F2 " << nv << " = kf2_sub(" << acc << ", " << t.second << ");\n";
+            else
+                o << ind << "const F2 " << nv << " = kf2_mac(" << acc << ", " << c << ", " << t.second << ");\n";
+            acc = nv;
+        }
+        if (acc.empty()) {
+            acc = var();
+            o << ind << "const F2 " << acc << " = kf2(0.0f);\n";
+        }
+        return acc;
+    }
+
     // Row of producer `in` needed by consumer k (image kimg) at primed tap
     // offset dyp, in iteration slot j.  `u` >= 0: the iteration index is the
     // compile-time constant u of a peeled edge iteration (rows relative to the
@@ -515,10 +619,12 @@ struct StreamGen {
                 s = sl(in, m + 2 * L - HY(in) - u, j);   // the iteration that computed row m of `in`
             }
         }
+        last_slot = s;
         std::vector<std::string> row;
         for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
         return row;
     }
+    int last_slot = 0;   // ring slot of the last tap_row (pair access in pair mode)
 
     // kernel k at iteration slot j: emits code, stores its V values into its
     // ring slot j, and memoises the unpacked values.
@@ -527,6 +633,16 @@ struct StreamGen {
         const Op &op = p->ops[k];
         const int img = p->n_inputs + k;
         std::vector<std::string> res(V);
+        if (pm && op.kind == POINT) {
+            const int ws = sl(img, 0, j);
+            for (int q = 0; q < V / 2; q++) {
+                std::vector<std::string> loads;
+                for (int in : op.inputs) loads.push_back(pval(in, sl(in, HY(img) - HY(in), j), q));
+                const std::string r = pe.emit2(o, op, loads, ind);
+                o << ind << ring(img, ws, q) << " = " << r << ";\n";
+            }
+            return;
+        }
         if (op.kind == POINT) {
             std::vector<std::vector<std::string>> ins;
             for (int in : op.inputs) {
@@ -550,6 +666,7 @@ struct StreamGen {
             if (sp.ok) {
                 // vertical pass in the lane's own columns, then horizontal taps
                 std::vector<std::pair<double, std::vector<std::string>>> rows;
+                std::vector<std::pair<double, int>> prow;   // pair mode: (coefficient, ring slot)
                 std::vector<double> cterms;   // coefficients of constant (exterior) rows
                 for (int dy = -ry; dy <= ry; dy++) {   // mask-row order in both directions (same rounding)
                     const int dyp = dir * dy;
@@ -558,7 +675,7 @@ struct StreamGen {
                     bool isc = false;
                     auto r = tap_row(img, op, in, dyp, j, u, isc, ind);
                     if (isc) cterms.push_back(c);
-                    else rows.push_back({c, r});
+                    else { rows.push_back({c, r}); prow.push_back({c, last_slot}); }
                 }
                 std::vector<std::string> vs(V);
                 std::string cst;
@@ -569,11 +686,22 @@ struct StreamGen {
                     o << ind << "const " << KV() << " " << cst << " = kf_mul1(" << (f32 ? fconst(cs) : iconst((long long)cs))
                       << ", " << cval(op) << ");\n";
                 }
-                for (int v = 0; v < V; v++) {
-                    std::vector<std::pair<double, std::string>> terms;
-                    for (auto &r : rows) terms.push_back({r.first, r.second[v]});
-                    if (!cst.empty()) terms.push_back({1.0, cst});
-                    vs[v] = lincomb(terms, ind);
+                if (pm) {
+                    for (int q = 0; q < V / 2; q++) {
+                        std::vector<std::pair<double, std::string>> terms;
+                        for (auto &r : prow) terms.push_back({r.first, pval(in, r.second, q)});
+                        if (!cst.empty()) terms.push_back({1.0, "kf2(" + cst + ")"});
+                        std::string pv = lincomb2(terms, ind);
+                        vs[2 * q] = pv + ".x";
+                        vs[2 * q + 1] = pv + ".y";
+                    }
+                } else {
+                    for (int v = 0; v < V; v++) {
+                        std::vector<std::pair<double, std::string>> terms;
+                        for (auto &r : rows) terms.push_back({r.first, r.second[v]});
+                        if (!cst.empty()) terms.push_back({1.0, cst});
+                        vs[v] = lincomb(terms, ind);
+                    }
                 }
                 // an exterior column of a CONSTANT consumer is c in every row: c * sum(col)
                 std::string csub;
@@ -610,6 +738,15 @@ struct StreamGen {
                 }
                 for (int v = 0; v < V; v++) acc[v] = lincomb(terms[v], ind);
             }
+            if (pm) {
+                const int ws = sl(img, 0, j);
+                for (int q = 0; q < V / 2; q++) {
+                    std::string pr = "make_float2(" + acc[2 * q] + ", " + acc[2 * q + 1] + ")";
+                    if (!op.prog.empty()) pr = pe.emit2(o, op, std::vector<std::string>{pr}, ind);
+                    o << ind << ring(img, ws, q) << " = " << pr << ";\n";
+                }
+                return;
+            }
             for (int v = 0; v < V; v++)
                 res[v] = op.prog.empty() ? acc[v] : pe.emit(o, op, k, std::vector<std::string>{acc[v]}, ind);
         }
@@ -643,10 +780,52 @@ struct StreamGen {
             std::string q = var();
             o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = " << (f32 ? "kf_ld4f(" : "kf_ld4u(")
               << ptr << ");\n";
-            for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
+            if (pm) {
+                o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
+                o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
+            } else {
+                for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
+            }
+        } else if (pm) {
+            for (int q = 0; q < V / 2; q++)
+                o << ind << ring(img, rs, q) << " = make_float2(__ldg(" << ptr << " + cl" << 2 * q << "), __ldg(" << ptr
+                  << " + cl" << 2 * q + 1 << "));\n";
         } else {
             for (int v = 0; v < V; v++)
                 o << ind << ring(img, rs, v) << " = __ldg(" << ptr << " + cl" << v << ");\n";
+        }
+    }
+
+    // primed-row expression -> clamped actual row of external image slot s
+    std::string row_of(int img, const std::string &it, const std::string &ind)
+    {
+        int s = slot.at(img);
+        std::string rp = "(ys - " + std::to_string(2 * si.L - HY(img)) + " + (" + it + "))";
+        std::string row = var();
+        o << ind << "const int " << row << " = min(max(" << (dir > 0 ? rp : "(H - 1 - " + rp + ")") << ", a.base["
+          << s << "]), a.rlast[" << s << "]);\n";
+        return row;
+    }
+    // shared-memory ring: start the copy of iteration `it`'s row into ring slot `ss`
+    void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
+    {
+        int s = slot.at(img);
+        std::string row = row_of(img, it, ind);
+        o << ind << "if ((" << it << ") < nit) kf_cp16(sr" << s << " + (" << ss << ") * 32, g" << s << " + " << row
+          << " * W);\n";
+    }
+    // shared-memory ring: read ring slot `ss` into register ring slot rs
+    void fetch(int img, const std::string &ss, int rs, const std::string &ind)
+    {
+        int s = slot.at(img);
+        std::string q = var();
+        o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = sr" << s << "[(" << ss << ") * 32];\n";
+        if (pm) {
+            o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
+            o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
+        } else {
+            const char *c[4] = {"x", "y", "z", "w"};
+            for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
         }
     }
 
@@ -657,7 +836,23 @@ struct StreamGen {
         val_memo.clear();
         shfl_memo.clear();
         o << ind.substr(2) << "{   // iteration " << uexpr << " + " << j << "\n";
-        for (int img : b.ext) load(img, sl(img, D, j), uexpr + " + " + std::to_string(j + D), ind);
+        if (si.sring) {
+            const int DS = si.DS;
+            std::string s_iss, s_get;
+            if (u >= 0) {   // peeled: static slots
+                s_iss = std::to_string((u + DS - 1) % DS);
+                s_get = std::to_string(u % DS);
+            } else {
+                s_iss = "kf_wrap_lt(qb + " + std::to_string(j + DS - 1) + ", " + std::to_string(DS) + ")";
+                s_get = "qb + " + std::to_string(j);
+            }
+            for (int img : b.ext) issue(img, s_iss, uexpr + " + " + std::to_string(j + DS - 1), ind);
+            o << ind << "kf_cp_commit();\n";
+            o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
+            for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
+        } else {
+            for (int img : b.ext) load(img, sl(img, D, j), uexpr + " + " + std::to_string(j + D), ind);
+        }
         for (int k : b.kernels) kernel(k, j, u, ind);
         const int simg = p->n_inputs + b.sink;
         const int ss = sl(simg, 0, j);
@@ -666,12 +861,13 @@ struct StreamGen {
         o << ind << "    const int yo = " << (dir > 0 ? "yp" : "H - 1 - yp") << ";\n";
         if (!si.vec) {
             for (int v = 0; v < V; v++) {
-                std::string val = f32 ? ring(simg, ss, v) : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
+                std::string val = f32 ? (pm ? value(simg, ss, v, ind) : ring(simg, ss, v))
+                                      : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
                 o << ind << "    if (x + " << v << " < a.fx1) gout[yo * W + " << v << "] = " << val << ";\n";
             }
         } else if (f32) {
             o << ind << "    kf_st4f(gout + yo * W";
-            for (int v = 0; v < V; v++) o << ", " << ring(simg, ss, v);
+            for (int v = 0; v < V; v++) o << ", " << (pm ? value(simg, ss, v, ind) : ring(simg, ss, v));
             o << ");\n";
         } else {
             o << ind << "    kf_st4u(gout + yo * W";
@@ -684,7 +880,7 @@ struct StreamGen {
             for (int k : b.kernels) imgs.insert(p->n_inputs + k);
             for (int img : imgs)
                 for (int a = ring_len(img) - 1; a >= 1; a--)
-                    for (int v = 0; v < V; v++) o << ind << ring(img, a, v) << " = " << ring(img, a - 1, v) << ";\n";
+                    for (int v = 0; v < NR(); v++) o << ind << ring(img, a, v) << " = " << ring(img, a - 1, v) << ";\n";
         }
         o << ind.substr(2) << "}\n";
     }
@@ -730,17 +926,30 @@ struct StreamGen {
         std::set<int> imgs(b.ext.begin(), b.ext.end());
         for (int k : b.kernels) imgs.insert(p->n_inputs + k);
         for (int img : imgs) {
-            o << "    " << RT();
+            o << "    " << RDT();
             bool first = true;
             for (int s = 0; s < ring_len(img); s++)
-                for (int v = 0; v < V; v++) {
-                    o << (first ? " " : ", ") << ring(img, s, v) << " = 0";
+                for (int v = 0; v < NR(); v++) {
+                    o << (first ? " " : ", ") << ring(img, s, v) << (pm ? " = kf2(0.0f)" : " = 0");
                     first = false;
                 }
             o << ";\n";
         }
-        for (int it = 0; it < D; it++)
-            for (int img : b.ext) load(img, si.rolled ? D - it : it % P, std::to_string(it), "    ");
+        if (si.sring) {
+            for (int img : b.ext) {
+                int s = slot.at(img);
+                o << "    " << (f32 ? "float4" : "uint4") << " *sr" << s << " = (" << (f32 ? "float4" : "uint4")
+                  << " *)(" << kernel_name(block) << "_ring + " << s * si.DS * 512 << ") + lane;\n";
+            }
+            for (int it = 0; it < si.DS - 1; it++) {
+                for (int img : b.ext) issue(img, std::to_string(it), std::to_string(it), "    ");
+                o << "    kf_cp_commit();\n";
+            }
+            o << "    int qb = 0;   // ring slot of the current iteration's row (multiple of the unroll)\n";
+        } else {
+            for (int it = 0; it < D; it++)
+                for (int img : b.ext) load(img, si.rolled ? D - it : it % P, std::to_string(it), "    ");
+        }
         o << "    " << RT() << " *__restrict__ gout = (" << RT() << " *)a.out + x - a.out_base * W;\n";
         int u0 = 0;
         if (ve) {
@@ -752,7 +961,9 @@ struct StreamGen {
             const int Q = (need + P - 1) / P * P;
             for (int u = 0; u < Q; u++) iteration(u % P, u, std::to_string(u - u % P), "      ");
             u0 = Q;
+            if (si.sring) o << "    qb = " << Q % si.DS << ";\n";
         }
+        const int step = si.rolled ? 1 : P;
         if (si.rolled) {
             o << "    #pragma unroll 1\n";
             o << "    for (int u = " << u0 << "; u < nit; u++) {\n";
@@ -761,12 +972,17 @@ struct StreamGen {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
             for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
         }
+        if (si.sring) o << "        qb += " << step << ";\n        if (qb == " << si.DS << ") qb = 0;\n";
         o << "    }\n}\n\n";
     }
 
     void run()
     {
         for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
+        pm = f32 && env_int("KFUSE_PAIRS", 1, 0, 1);
+        if (si.sring)
+            o << "__shared__ __align__(16) unsigned char " << kernel_name(block) << "_ring[" << si.ring_bytes
+              << "];   // per-warp input row rings (one warp per CTA)\n\n";
         // Variants (the variant is CTA-uniform):
         //   interior strip, interior chunk   -- the hot loop, no border logic
         //   interior strip, edge chunk       -- + lane selects at x == 0 / x == W-4
@@ -855,8 +1071,11 @@ static Separable factor(const Op &op, bool integer)
         for (auto &r : row) r = -r;
     }
     s.ok = true;
-    for (int j = 0; j < mh; j++) s.col.push_back((double)col[j]);
-    for (int i = 0; i < mw; i++) s.row.push_back((double)row[i] * scale);
+    // the power-of-two scale goes to the column factor: the vertical pass runs
+    // on packed pixel pairs, the horizontal one per pixel, so the horizontal
+    // pass keeps its unit coefficients (one multiply fewer per pixel)
+    for (int j = 0; j < mh; j++) s.col.push_back((double)col[j] * scale);
+    for (int i = 0; i < mw; i++) s.row.push_back((double)row[i]);
     return s;
 }
 
@@ -893,14 +1112,28 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
         (ext ? maxdepth_ext : maxdepth) = std::max(ext ? maxdepth_ext : maxdepth, kv.second);
     }
-    // prefetch distance and ring period: P >= depth_ext + D, P >= every depth
+    // input feed: a cp.async shared-memory ring of DS rows per external image
+    // (128-bit rows), else register prefetch D iterations ahead.  Ring period
+    // P >= every depth (+ D for register-prefetched external images).
     si.D = env_int("KFUSE_PREFETCH", 4, 1, 16);
-    si.P = std::max(maxdepth, maxdepth_ext + si.D);
+    si.sring = si.vec && env_int("KFUSE_SRING", 1, 0, 1) && !b.ext.empty();
+    if (si.sring) {
+        si.P = std::max(maxdepth, maxdepth_ext);
+        const int want = env_int("KFUSE_SMEM_ROWS", 12, 2, 64);
+        const int cap = 32768 / (512 * (int)b.ext.size());   // <= 32 KB of ring per warp
+        int DS = std::max(want, si.P + 1);
+        DS = (DS + si.P - 1) / si.P * si.P;
+        while (DS > cap && DS - si.P >= si.P + 1) DS -= si.P;
+        if (DS > cap || DS < 2) si.sring = false;
+        si.DS = DS;
+        si.ring_bytes = (int)b.ext.size() * DS * 512;
+    }
+    if (!si.sring) si.P = std::max(maxdepth, maxdepth_ext + si.D);
     // register estimate: live ring values (depth per image, D prefetched rows)
     int live = 0;
     for (auto &kv : si.depth) {
         bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
-        live += (kv.second + (ext ? si.D : 0)) * kStreamV;
+        live += (kv.second + (ext && !si.sring ? si.D : 0)) * kStreamV;
     }
     si.live_regs = live;
     // code size: scalar operations of one iteration (one body copy)

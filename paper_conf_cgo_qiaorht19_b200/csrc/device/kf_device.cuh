@@ -194,3 +194,51 @@ __device__ __forceinline__ I4 kf_shdn(I4 v, int d)
 // first product of an accumulation (mask coefficient m)
 __device__ __forceinline__ float kf_mul1(float m, float v) { return m * v; }
 __device__ __forceinline__ I4 kf_mul1(int m, I4 v) { return I4{m * v.x, m * v.y, m * v.z, m * v.w}; }
+
+// ------------------------------------------------ packed f32x2 (sm_100a)
+// Two adjacent pixels of a lane as one 64-bit register pair: FFMA2 / FADD2 /
+// FMUL2 issue one instruction for both.  Operations without a
+// packed form run per component.
+typedef float2 F2;
+__device__ __forceinline__ F2 kf2(float a) { return make_float2(a, a); }
+__device__ __forceinline__ F2 kf2_add(F2 a, F2 b) { return __fadd2_rn(a, b); }
+__device__ __forceinline__ F2 kf2_sub(F2 a, F2 b) { return __fadd2_rn(a, make_float2(-b.x, -b.y)); }
+__device__ __forceinline__ F2 kf2_mul(F2 a, F2 b) { return __fmul2_rn(a, b); }
+__device__ __forceinline__ F2 kf2_fma(F2 a, F2 b, F2 c) { return __ffma2_rn(a, b, c); }          // a*b + c
+__device__ __forceinline__ F2 kf2_fms(F2 a, F2 b, F2 c) { return __ffma2_rn(a, b, make_float2(-c.x, -c.y)); }  // a*b - c
+__device__ __forceinline__ F2 kf2_nfma(F2 a, F2 b, F2 c) { return __ffma2_rn(make_float2(-a.x, -a.y), b, c); }  // c - a*b
+__device__ __forceinline__ F2 kf2_mac(F2 acc, float m, F2 v) { return __ffma2_rn(v, make_float2(m, m), acc); }
+__device__ __forceinline__ F2 kf2_mul1(float m, F2 v) { return __fmul2_rn(v, make_float2(m, m)); }
+__device__ __forceinline__ F2 kf2_div(F2 a, F2 b) { return make_float2(a.x / b.x, a.y / b.y); }
+__device__ __forceinline__ F2 kf2_min(F2 a, F2 b) { return make_float2(fminf(a.x, b.x), fminf(a.y, b.y)); }
+__device__ __forceinline__ F2 kf2_max(F2 a, F2 b) { return make_float2(fmaxf(a.x, b.x), fmaxf(a.y, b.y)); }
+__device__ __forceinline__ F2 kf2_abs(F2 a) { return make_float2(fabsf(a.x), fabsf(a.y)); }
+__device__ __forceinline__ F2 kf2_neg(F2 a) { return make_float2(-a.x, -a.y); }
+__device__ __forceinline__ F2 kf2_sqrt(F2 a) { return make_float2(sqrtf(a.x), sqrtf(a.y)); }
+__device__ __forceinline__ F2 kf2_exp(F2 a) { return make_float2(expf(a.x), expf(a.y)); }
+__device__ __forceinline__ F2 kf2_log(F2 a) { return make_float2(logf(a.x), logf(a.y)); }
+__device__ __forceinline__ F2 kf2_pow(F2 a, F2 b) { return make_float2(powf(a.x, b.x), powf(a.y, b.y)); }
+__device__ __forceinline__ F2 kf2_clamp(F2 a, F2 lo, F2 hi)
+{
+    return make_float2(fminf(fmaxf(a.x, lo.x), hi.x), fminf(fmaxf(a.y, lo.y), hi.y));
+}
+__device__ __forceinline__ F2 kf2_sel_gt(F2 a, F2 b, F2 c, F2 d)
+{
+    return make_float2(a.x > b.x ? c.x : d.x, a.y > b.y ? c.y : d.y);
+}
+
+// ------------------------------------------- asynchronous row ring (cp.async)
+// Each streaming warp keeps DS input rows (512 B each) in flight in a shared
+// memory ring: 16 B per lane per row via cp.async (LDGSTS), one commit group
+// per row, consumed DS-1 groups later.
+__device__ __forceinline__ void kf_cp16(void *smem, const void *gmem)
+{
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void kf_cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N> __device__ __forceinline__ void kf_cp_wait()
+{
+    asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ int kf_wrap_lt(int x, int n) { return x >= n ? x - n : x; }

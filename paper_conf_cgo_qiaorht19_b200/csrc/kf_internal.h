@@ -122,7 +122,7 @@ BlockInfo analyse_block(const kf_pipeline *p, const std::vector<int> &kernels);
 // codegen.cpp
 constexpr int kStreamV = 4;                              // pixels per lane of the interior path
 constexpr int kThreads = 32;                             // threads per CTA (both paths): one warp
-constexpr int kMinCtasPerSm = 16;                        // __launch_bounds__ min blocks (<= 128 regs)
+constexpr int kMinCtasPerSm = 12;                        // __launch_bounds__ min blocks (<= 168 regs)
 constexpr int KF_MAX_IMG_HOST = 16;                      // = KF_MAX_IMG of kf_device.cuh
 constexpr int kFrameTiles[2][2] = {{32, 8}, {8, 32}};    // frame tile shapes (w, h)
 
@@ -141,6 +141,9 @@ struct StreamInfo {
     int D = 4;                    // prefetch distance (iterations)
     int live_regs = 0;            // estimate of ring registers
     bool rolled = false;          // one loop-body copy + ring shifts (big blocks)
+    bool sring = false;           // external rows fed by a cp.async shared-memory ring
+    int DS = 0;                   // rows in that ring (multiple of P)
+    int ring_bytes = 0;           // its shared memory per warp
     long long iter_ops = 0;       // scalar operations per iteration (code-size estimate)
     bool edge_v = false;          // top/bottom image edges handled by edge strips
     bool edge_l = false, edge_r = false;   // left/right image edges handled by edge chunks

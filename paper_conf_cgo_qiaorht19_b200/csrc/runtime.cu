@@ -296,7 +296,10 @@ static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlo
         const int last = Hf - (nst - 1) * S;
         const long long items = (long long)a.n_chunks * nst;
         const long long waves = (items + slots - 1) / slots;
-        auto iters = [&](int rows) { return (long long)(rows + 2 * si.L + si.P - 1) / si.P * si.P; };
+        // per item: warm-up 2L rows, rounding to the unroll P, the row feed's
+        // prefetch depth (ring rows / register prefetch) and the start-up latency
+        const int over = (si.sring ? si.DS : si.D) + 4;
+        auto iters = [&](int rows) { return (long long)(rows + 2 * si.L + si.P - 1) / si.P * si.P + over; };
         // the wave containing the long last strip bounds the time
         const long long cost = (waves - 1) * iters(S) + iters(last);
         if (best < 0 || cost < best) { best = cost; best_S = S; }

@@ -139,7 +139,7 @@ class Pipeline:
         self.outputs: list[int] = []
 
     def __del__(self):
-        if getattr(self, "h", None):
+        if getattr(self, "h", None) and lib is not None:
             lib.kf_pipeline_destroy(self.h)
             self.h = None
 
@@ -216,7 +216,7 @@ class Plan:
         self.pipe, self.h = pipe, h
 
     def __del__(self):
-        if getattr(self, "h", None):
+        if getattr(self, "h", None) and lib is not None:
             lib.kf_plan_destroy(self.h)
             self.h = None
 

@@ -36,12 +36,13 @@ def child(cfg: str, plan_kind: str, steps: int) -> None:
     with torch.cuda.graph(g, stream=s):
         for i in range(steps):
             plan.run([ins[i % 4]], [outs[i % 4]], s)
-    g.replay()
-    torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(s)
-    g.replay()
-    e1.record(s)
+    with torch.cuda.stream(s):            # replay() launches on the current stream
+        g.replay()
+        torch.cuda.synchronize()
+        e0.record(s)
+        g.replay()
+        e1.record(s)
     torch.cuda.synchronize()
     us = e0.elapsed_time(e1) / steps * 1e3
     print(json.dumps({"us": round(us, 2), "gpx_s": round(W * H / us / 1e3, 1)}))
