@@ -192,6 +192,22 @@ def deep10(width: int, height: int, mode: str = "mirror") -> dict:
     return p.spec()
 
 
+def copy(width: int, height: int, mode: str = "clamp") -> dict:
+    """Diagnostic: one point kernel out = in (the streaming path's memory-side ceiling)."""
+    p = Pipeline("copy", width, height, "f32")
+    i = p.input()
+    p.output(p.point("copy", [i], [L(0)]))
+    return p.spec()
+
+
+def blur(width: int, height: int, mode: str = "clamp") -> dict:
+    """Diagnostic: one 3x3 Gaussian local kernel."""
+    p = Pipeline("blur", width, height, "f32")
+    i = p.input()
+    p.output(p.local("blur", i, GAUSS3_N, mode))
+    return p.spec()
+
+
 def fig4(mode: str = "clamp") -> dict:
     """Fig. 4: two unnormalised 3x3 Gaussian local kernels on a 5x5 image."""
     p = Pipeline("fig4", 5, 5, "f32")
@@ -294,6 +310,8 @@ WORKLOADS = {
     "sobel": sobel,
     "enhance": enhance,
     "deep10": deep10,
+    "copy": copy,
+    "blur": blur,
 }
 
 # BASELINE.json configs: (workload, W, H, seed)

@@ -369,12 +369,15 @@ struct FrameGen {
         if (smem > 48 * 1024) fail(KF_ERR_ARG, "fused block needs more than 48 KB of shared memory");
         // dispatcher for frame CTAs
         o << "__device__ __forceinline__ void " << kernel_name(block) << "_frame(const KfArgs &a, int cta)\n{\n";
+        int off = 0;   // staged tiles live in the block's shared buffer (shared with the interior rings)
         for (auto &g : groups)
             for (int k : g) {
                 int n = 0;
                 for (int s = 0; s < 2; s++)
                     n = std::max(n, (kFrameTiles[s][0] + 2 * b.hx.at(k)) * (kFrameTiles[s][1] + 2 * b.hy.at(k)));
-                o << "    __shared__ " << (f32 ? "float " : "unsigned ") << smem_name(k) << "[" << n << "];\n";
+                o << "    " << (f32 ? "float" : "unsigned") << " *" << smem_name(k) << " = (" << (f32 ? "float" : "unsigned")
+                  << " *)(" << kernel_name(block) << "_smem + " << off << ");\n";
+                off += n * 4;
             }
         std::string sargs;
         for (auto &g : groups)
@@ -434,6 +437,8 @@ struct StreamGen {
     int dir = 1;
     bool el = false, er = false;
     bool pm = false;   // f32 values kept as packed pixel pairs (F2) for column-local math
+    bool runptr = false;   // steady-state loop uses running row pointers (set per variant)
+    bool vedge = false;    // variant starts at an image edge (peeled iterations remap taps)
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
@@ -607,7 +612,7 @@ struct StreamGen {
         const int L = si.L;
         int s = sl(in, HY(kimg) - HY(in) + dyp, j);
         is_const = false;
-        if (u >= 0) {
+        if (u >= 0 && vedge) {
             const int rk = u - 2 * L + HY(kimg);   // consumer row (primed, 0 = edge row)
             const int rr = rk + dyp;
             if (rr < 0 && rk >= 0) {
@@ -810,6 +815,11 @@ struct StreamGen {
     void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
     {
         int s = slot.at(img);
+        if (runptr) {   // steady state: running row pointer (rows stay inside [base, rlast])
+            o << ind << "if ((" << it << ") < nit) kf_cp16(sr" << s << " + (" << ss << ") * 32, ip" << s << ");\n";
+            o << ind << "ip" << s << " += dW;\n";
+            return;
+        }
         std::string row = row_of(img, it, ind);
         o << ind << "if ((" << it << ") < nit) kf_cp16(sr" << s << " + (" << ss << ") * 32, g" << s << " + " << row
           << " * W);\n";
@@ -843,7 +853,7 @@ struct StreamGen {
                 s_iss = std::to_string((u + DS - 1) % DS);
                 s_get = std::to_string(u % DS);
             } else {
-                s_iss = "kf_wrap_lt(qb + " + std::to_string(j + DS - 1) + ", " + std::to_string(DS) + ")";
+                s_iss = j == 0 ? "qprev" : "qb + " + std::to_string(j - 1);
                 s_get = "qb + " + std::to_string(j);
             }
             for (int img : b.ext) issue(img, s_iss, uexpr + " + " + std::to_string(j + DS - 1), ind);
@@ -853,28 +863,44 @@ struct StreamGen {
         } else {
             for (int img : b.ext) load(img, sl(img, D, j), uexpr + " + " + std::to_string(j + D), ind);
         }
-        for (int k : b.kernels) kernel(k, j, u, ind);
+        for (int k : b.kernels) {
+            // warm-up (peeled) iteration: kernel k is first needed at iteration 2L - 2 HY(k)
+            if (u >= 0 && u < 2 * L - 2 * HY(p->n_inputs + k)) continue;
+            kernel(k, j, u, ind);
+        }
         const int simg = p->n_inputs + b.sink;
         const int ss = sl(simg, 0, j);
-        o << ind << "const int yp = ys - " << 2 * L << " + " << uexpr << " + " << j << ";\n";
-        o << ind << "if (xst && yp >= ys && yp < ye) {\n";
-        o << ind << "    const int yo = " << (dir > 0 ? "yp" : "H - 1 - yp") << ";\n";
-        if (!si.vec) {
+        const bool store = !(u >= 0 && u < 2 * L);   // warm-up iterations store nothing
+        std::string orow;   // output row pointer expression
+        if (!store) {
+            o << ind << "{\n";
+        } else if (runptr) {
+            o << ind << "if (xst && (unsigned)(" << uexpr << " + " << j - 2 * L << ") < (unsigned)(ye - ys)) {\n";
+            orow = "op";
+        } else {
+            o << ind << "const int yp = ys - " << 2 * L << " + " << uexpr << " + " << j << ";\n";
+            o << ind << "if (xst && yp >= ys && yp < ye) {\n";
+            o << ind << "    const int yo = " << (dir > 0 ? "yp" : "H - 1 - yp") << ";\n";
+            orow = "gout + yo * W";
+        }
+        if (!store) {
+        } else if (!si.vec) {
             for (int v = 0; v < V; v++) {
                 std::string val = f32 ? (pm ? value(simg, ss, v, ind) : ring(simg, ss, v))
                                       : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
-                o << ind << "    if (x + " << v << " < a.fx1) gout[yo * W + " << v << "] = " << val << ";\n";
+                o << ind << "    if (x + " << v << " < a.fx1) (" << orow << ")[" << v << "] = " << val << ";\n";
             }
         } else if (f32) {
-            o << ind << "    kf_st4f(gout + yo * W";
+            o << ind << "    kf_st4f(" << orow;
             for (int v = 0; v < V; v++) o << ", " << (pm ? value(simg, ss, v, ind) : ring(simg, ss, v));
             o << ");\n";
         } else {
-            o << ind << "    kf_st4u(gout + yo * W";
+            o << ind << "    kf_st4u(" << orow;
             for (int v = 0; v < V; v++) o << ", kf_pack(" << val_memo[std::make_tuple(simg, ss, v)] << ")";
             o << ");\n";
         }
         o << ind << "}\n";
+        if (runptr) o << ind << "op += dW;\n";
         if (si.rolled) {   // age every ring by one row
             std::set<int> imgs(b.ext.begin(), b.ext.end());
             for (int k : b.kernels) imgs.insert(p->n_inputs + k);
@@ -904,8 +930,10 @@ struct StreamGen {
         o << "    const int x = a.fx0 + (chunk * " << 32 - 2 * HL << " + lane - " << HL << ") * " << V << ";\n";
         o << "    const bool xst = lane >= " << HL << " && lane < " << 32 - HL << " && x < a.fx1;\n";
         // strip bounds in primed (streaming-direction) rows
-        o << "    const int ys0 = a.fy0 + strip * a.strip;\n";
-        o << "    const int ye0 = strip == a.n_strips - 1 ? a.fy1 : ys0 + a.strip;   // the last strip takes the rest\n";
+        // balanced strips: strip i covers rows [fy0 + i*Hf/ns, fy0 + (i+1)*Hf/ns)
+        o << "    const int Hf = a.fy1 - a.fy0;\n";
+        o << "    const int ys0 = a.fy0 + (int)((long long)strip * Hf / a.n_strips);\n";
+        o << "    const int ye0 = a.fy0 + (int)((long long)(strip + 1) * Hf / a.n_strips);\n";
         if (dir > 0) {
             o << "    const int ys = ys0, ye = ye0;\n";
         } else {
@@ -939,7 +967,7 @@ struct StreamGen {
             for (int img : b.ext) {
                 int s = slot.at(img);
                 o << "    " << (f32 ? "float4" : "uint4") << " *sr" << s << " = (" << (f32 ? "float4" : "uint4")
-                  << " *)(" << kernel_name(block) << "_ring + " << s * si.DS * 512 << ") + lane;\n";
+                  << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 << ") + lane;\n";
             }
             for (int it = 0; it < si.DS - 1; it++) {
                 for (int img : b.ext) issue(img, std::to_string(it), std::to_string(it), "    ");
@@ -952,37 +980,58 @@ struct StreamGen {
         }
         o << "    " << RT() << " *__restrict__ gout = (" << RT() << " *)a.out + x - a.out_base * W;\n";
         int u0 = 0;
-        if (ve) {
-            // peeled iterations in which some tap row lies beyond the edge
-            int need = 0;
+        // peeled iterations: the 2L warm-up iterations (only the kernels whose rows
+        // are needed run) and, at an image edge, those in which some tap row lies
+        // beyond the edge (remapped statically)
+        int need = si.rolled ? 0 : 2 * L;
+        vedge = ve;
+        if (ve)
             for (int k : b.kernels)
                 if (p->ops[k].kind == LOCAL)
                     need = std::max(need, 2 * L - HY(p->n_inputs + k) + p->ops[k].ry());
+        if (need > 0) {
             const int Q = (need + P - 1) / P * P;
             for (int u = 0; u < Q; u++) iteration(u % P, u, std::to_string(u - u % P), "      ");
             u0 = Q;
             if (si.sring) o << "    qb = " << Q % si.DS << ";\n";
         }
+        vedge = false;
         const int step = si.rolled ? 1 : P;
+        // steady state: running pointers for the next row to fetch into the ring and
+        // the next output row (valid when the ring is deep enough that every row it
+        // fetches after the prologue lies inside [base, rlast])
+        const bool rp_ok = si.sring && si.DS - 1 >= 2 * L;
+        if (rp_ok) {
+            o << "    const int dW = " << (dir > 0 ? "W" : "-W") << ";\n";
+            for (int img : b.ext) {
+                int s = slot.at(img);
+                std::string row = row_of(img, std::to_string(u0 + si.DS - 1), "    ");
+                o << "    const " << RT() << " *__restrict__ ip" << s << " = g" << s << " + " << row << " * W;\n";
+            }
+            std::string yp0 = "(ys - " + std::to_string(2 * L - u0) + ")";
+            o << "    " << RT() << " *__restrict__ op = gout + " << (dir > 0 ? yp0 : "(H - 1 - " + yp0 + ")") << " * W;\n";
+            runptr = true;
+        }
         if (si.rolled) {
             o << "    #pragma unroll 1\n";
             o << "    for (int u = " << u0 << "; u < nit; u++) {\n";
+            if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
             iteration(0, -1, "u", "        ");
         } else {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
+            if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
             for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
         }
         if (si.sring) o << "        qb += " << step << ";\n        if (qb == " << si.DS << ") qb = 0;\n";
         o << "    }\n}\n\n";
+        runptr = false;
     }
 
     void run()
     {
         for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
         pm = f32 && env_int("KFUSE_PAIRS", 1, 0, 1);
-        if (si.sring)
-            o << "__shared__ __align__(16) unsigned char " << kernel_name(block) << "_ring[" << si.ring_bytes
-              << "];   // per-warp input row rings (one warp per CTA)\n\n";
+
         // Variants (the variant is CTA-uniform):
         //   interior strip, interior chunk   -- the hot loop, no border logic
         //   interior strip, edge chunk       -- + lane selects at x == 0 / x == W-4
@@ -1194,6 +1243,17 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
             for (size_t i = 0; i < p->ops[k].lut.size(); i++) o << (i ? "," : "") << p->ops[k].lut[i];
             o << "};\n";
         }
+    // one shared buffer per CTA: the frame path's staged tiles OR the interior
+    // warp's input row rings (a CTA runs exactly one of the two paths)
+    int frame_bytes = 0;
+    for (int k : b.staged) {
+        int n = 0;
+        for (int s = 0; s < 2; s++)
+            n = std::max(n, (kFrameTiles[s][0] + 2 * b.hx.at(k)) * (kFrameTiles[s][1] + 2 * b.hy.at(k)));
+        frame_bytes += n * 4;
+    }
+    const int smem_bytes = std::max(16, std::max(frame_bytes, si.ok && si.sring ? si.ring_bytes : 0));
+    o << "__shared__ __align__(16) unsigned char " << kernel_name(block) << "_smem[" << smem_bytes << "];\n\n";
     FrameGen fg(p, b, block, o);
     fg.run();
     if (si.ok) {

@@ -282,31 +282,30 @@ static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlo
     a.n_chunks = (fx1 - fx0 + chunk_w - 1) / chunk_w;
     const int Hf = fy1 - fy0;
     const long long slots = (long long)cb.num_sms * cb.ctas_per_sm;   // resident single-warp CTAs per wave
-    // n_strips = floor(Hf / S): strips of S rows, the last one takes the rest
-    // (< 2S).  Edge strips must be at least L rows so that no interior strip
-    // reads beyond the image; a top and a bottom edge need two strips.
+    // ns balanced strips of floor/ceil(Hf/ns) rows.  Edge strips must be at
+    // least L rows so that no interior strip reads beyond the image; a top and
+    // a bottom edge need two strips.  Cost (fitted to B200 sweeps, DESIGN.md
+    // §5.4): (iterations of one item + 2) x (waves + 1/2), iterations = rows +
+    // 2L warm-up rounded up to the unroll P.  Several waves of short items
+    // beat one wave of long ones: the hardware refills freed CTA slots, which
+    // desynchronises the warps' load bursts and shortens the tail.
     const int min_strips = top && bot ? 2 : 1;
     const int smin = top || bot ? std::max(1, si.L) : 1;
-    long long best = -1;
-    int best_S = Hf / min_strips;
+    auto iters = [&](int rows) { return (double)((rows + 2 * si.L + si.P - 1) / si.P * si.P + 2); };
+    double best = -1.0;
+    int best_ns = min_strips;
     for (int ns = min_strips; ns <= std::max(min_strips, Hf / smin); ns++) {
-        const int S = Hf / ns;
-        if (ns > min_strips && Hf / (ns - 1) == S) continue;
-        const int nst = Hf / S;
-        const int last = Hf - (nst - 1) * S;
-        const long long items = (long long)a.n_chunks * nst;
-        const long long waves = (items + slots - 1) / slots;
-        // per item: warm-up 2L rows, rounding to the unroll P, the row feed's
-        // prefetch depth (ring rows / register prefetch) and the start-up latency
-        const int over = (si.sring ? si.DS : si.D) + 4;
-        auto iters = [&](int rows) { return (long long)(rows + 2 * si.L + si.P - 1) / si.P * si.P + over; };
-        // the wave containing the long last strip bounds the time
-        const long long cost = (waves - 1) * iters(S) + iters(last);
-        if (best < 0 || cost < best) { best = cost; best_S = S; }
+        const int S = (Hf + ns - 1) / ns;
+        const long long items = (long long)a.n_chunks * ns;
+        const double w = (double)items / (double)slots;
+        const double cost = iters(S) * (w + 0.5);
+        if (best < 0 || cost < best - 1e-9) { best = cost; best_ns = ns; }
         if (items > 64 * slots) break;
     }
-    a.strip = best_S;
-    a.n_strips = Hf / best_S;
+    if (const int force = env_int("KFUSE_NSTRIPS", 0, 0, 1 << 20))   // tuning / diagnostics
+        best_ns = std::max(min_strips, std::min(force, std::max(min_strips, Hf / smin)));
+    a.n_strips = best_ns;
+    a.strip = (Hf + best_ns - 1) / best_ns;
     a.n_items = a.n_chunks * a.n_strips;
     return (unsigned)(cta + a.n_items);
 }

@@ -20,7 +20,11 @@ def child(cfg: str, plan_kind: str, steps: int) -> None:
     from kf_inputs import gen
     from kf_inputs import pipelines as P
     from paper_conf_cgo_qiaorht19_b200 import kfuse as K
-    spec, seed = P.config(cfg)
+    if ":" in cfg:   # workload:W:H
+        wl, w, h = cfg.split(":")
+        spec, seed = P.WORKLOADS[wl](int(w), int(h)), 1
+    else:
+        spec, seed = P.config(cfg)
     W, H = spec["width"], spec["height"]
     host = gen.image(spec["dtype"], seed, W, H)
     ins = [torch.from_numpy(host).cuda() for _ in range(4)]
