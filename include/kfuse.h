@@ -160,6 +160,19 @@ kf_status kf_mark_output(kf_pipeline *p, int32_t image_id);
 /* ---- planning (host only; freezes the graph) ---------------------------- */
 /* Alg. 1 GetLegalPartitions with the benefit model. */
 kf_status kf_plan_fusion(kf_pipeline *p, const kf_model_params *m, kf_plan **out);
+/* The "basic" fusion of the authors' previous work [12], the paper's
+ * comparison column: only
+ * point-to-point, local-to-point and point-to-local fusion, shared inputs
+ * (Fig. 2b) rejected as external.  Greedy pair-wise merging by decreasing
+ * edge benefit under IsLegal plus the basic rules (R-18).  Same
+ * weights, output and ownership as kf_plan_fusion. */
+kf_status kf_plan_basic(kf_pipeline *p, const kf_model_params *m, kf_plan **out);
+/* Exact planner: the partition into IsLegal blocks with the
+ * maximum total weight of the edges inside blocks (Eq. 1, lexicographic
+ * (q, eps)), by subset DP in O(3^n) -- the exhaustive search the paper rules
+ * out for large graphs.  KF_ERR_ARG for more than 16
+ * kernels.  Same output and ownership as kf_plan_fusion. */
+kf_status kf_plan_exact(kf_pipeline *p, const kf_model_params *m, kf_plan **out);
 /* Every kernel its own block: the unfused GPU baseline. */
 kf_status kf_plan_unfused(kf_pipeline *p, kf_plan **out);
 /* Caller-chosen partition: block_of_kernel[k] = block label (any ints).  Every
@@ -213,8 +226,15 @@ kf_status kf_run(kf_pipeline *p, const kf_plan *plan, const void *const *d_input
                  void *const *d_outputs, int32_t n_out, void *stream);
 
 /* End-to-end call with HOST buffers: copies inputs host->device, runs, copies
- * outputs device->host, synchronises `stream`.  Host buffers should be pinned
- * for full PCIe bandwidth.  Device staging buffers are owned by the pipeline. */
+ * outputs device->host, synchronises `stream`.  The image is processed in up to
+ * 8 row bands on three engines: the H2D copy of band k+1's input rows, the
+ * kernels of band k (kf_run_band semantics: border modes act at the global
+ * edges, so the result equals kf_run's bit for bit) and the D2H copy of band
+ * k-1's output rows overlap.  REPEAT plans run as one band.  Host buffers
+ * (same layout as kf_run's device buffers) should be pinned for full
+ * host-link bandwidth and overlap; pageable buffers work but serialise the
+ * copies.  Device staging buffers, the two copy streams and their events are
+ * owned by the pipeline.  Work already queued on `stream` precedes the copies. */
 kf_status kf_run_host(kf_pipeline *p, const kf_plan *plan, const void *const *h_inputs, int32_t n_in,
                       void *const *h_outputs, int32_t n_out, void *stream);
 

@@ -15,6 +15,9 @@ Contents, each in the paper's notation:
   get_legal_partitions()  Alg. 1 (PAPER.md:717-769)
   brute_force()   exact maximum of Eq. 1 over all partitions into legal blocks
                   (the paper's "exhaustive search")
+  basic_fusion()  the "basic" fusion of the authors' previous work [12], the
+                  comparison column of Table I,
+                  reading R-18
 
 Parity unpinned (R-4, R-7): the local-to-local locality gain of Eq. 3
 (garbled, read as IS*tg/ts) and the B200 profile's STAGED recompute factor have
@@ -370,6 +373,72 @@ def brute_force(spec: dict, m: Model = PAPER_PROFILE) -> tuple[tuple, list]:
 
     rec2(0)
     return best[0], best[1]
+
+
+# ------------------------------------------------------ basic fusion [12]
+
+
+def basic_legal(g: Graph, P: set, m: Model, info: dict) -> bool:
+    """Reading R-18 of [12] as the paper describes it ("fusion
+    ... only for point operator related fusion, namely point-to-point,
+    local-to-point, and point-to-local"; Sobel's local-to-local
+    and Unsharp's shared input "are rejected by the basic kernel fusion
+    algorithm"): IsLegal, plus exactly one source kernel, no other kernel reads an
+    image from outside P (a shared input counts as external), and no local kernel
+    has a local kernel upstream inside P."""
+    if len(P) == 1:
+        return True
+    if not is_legal(g, P, m, info):
+        return False
+    sources = [k for k in P if not any(p in P for p in g.producers[k])]
+    if len(sources) != 1:
+        return False
+    for k in P:
+        if k == sources[0]:
+            continue
+        for img in g.inputs[k]:
+            if not (img >= g.n_inputs and (img - g.n_inputs) in P):
+                return False
+    for k in P:
+        if g.kind[k] != "local":
+            continue
+        # every kernel upstream of k inside P
+        up, stack = set(), [p for p in g.producers[k] if p in P]
+        while stack:
+            u = stack.pop()
+            if u in up:
+                continue
+            up.add(u)
+            stack += [p for p in g.producers[u] if p in P]
+        if any(g.kind[u] == "local" for u in up):
+            return False
+    return True
+
+
+def basic_fusion(spec: dict, m: Model = PAPER_PROFILE) -> list:
+    """Pair-wise greedy fusion of [12] (reading R-18): visit the profitable edges by
+    decreasing benefit w (ties: lower producer, then lower consumer); merge the two
+    blocks the edge joins when their union is basic-legal; repeat full passes until
+    nothing merges.  Returns the blocks sorted by their largest kernel."""
+    g = graph(spec)
+    info = edge_weights(g, m)
+    block = {k: {k} for k in range(g.n)}          # kernel -> its block (shared sets)
+    order = sorted((e for e in info.values() if e.profitable), key=lambda e: (-e.w, e.ks, e.kd))
+    changed = True
+    while changed:
+        changed = False
+        for e in order:
+            a, b = block[e.ks], block[e.kd]
+            if a is b:
+                continue
+            u = a | b
+            if not basic_legal(g, u, m, info):
+                continue
+            for k in u:
+                block[k] = u
+            changed = True
+    blocks = {id(b): sorted(b) for b in block.values()}
+    return sorted(blocks.values(), key=max)
 
 
 def min_cut_brute(g: Graph, P: list, info: dict) -> tuple:

@@ -200,6 +200,22 @@ kf_status kf_plan_fusion(kf_pipeline *p, const kf_model_params *m, kf_plan **out
     });
 }
 
+kf_status kf_plan_basic(kf_pipeline *p, const kf_model_params *m, kf_plan **out)
+{
+    return guard([&] {
+        if (!p || !m || !out) fail(KF_ERR_ARG, "null pointer");
+        *out = plan_basic(p, *m);
+    });
+}
+
+kf_status kf_plan_exact(kf_pipeline *p, const kf_model_params *m, kf_plan **out)
+{
+    return guard([&] {
+        if (!p || !m || !out) fail(KF_ERR_ARG, "null pointer");
+        *out = plan_exact(p, *m);
+    });
+}
+
 kf_status kf_plan_unfused(kf_pipeline *p, kf_plan **out)
 {
     return guard([&] {

@@ -36,7 +36,16 @@
 
 namespace kf {
 
-std::string kernel_name(int block) { return "kf_b" + std::to_string(block); }
+// Entry-point name: block index, sink kernel and block size, so that launch
+// lists of different plans of one pipeline tell their kernels apart.
+std::string kernel_name(const BlockInfo &b, int block)
+{
+    return "kf_b" + std::to_string(block) + "_k" + std::to_string(b.sink) + "n" + std::to_string(b.kernels.size());
+}
+
+namespace {
+std::string kernel_name(int block) { return "kf_b" + std::to_string(block); }   // prefix of the device helpers
+}  // namespace
 
 namespace {
 
@@ -1260,7 +1269,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
         StreamGen sg(p, b, si, block, o);
         sg.run();
     }
-    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << env_int("KFUSE_MINCTAS", kMinCtasPerSm, 1, 32) << ") " << kernel_name(block)
+    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << env_int("KFUSE_MINCTAS", kMinCtasPerSm, 1, 32) << ") " << kernel_name(b, block)
       << "(const __grid_constant__ KfArgs a)\n{\n";
     o << "    const int cta = blockIdx.x;\n";
     o << "    if (cta < a.frame_ctas) { " << kernel_name(block) << "_frame(a, cta); return; }\n";

@@ -114,6 +114,8 @@ std::vector<std::vector<int>> producers(const kf_pipeline *p);   // kernel -> pr
 
 // planner.cpp
 kf_plan *plan_fusion(kf_pipeline *p, const kf_model_params &m);
+kf_plan *plan_basic(kf_pipeline *p, const kf_model_params &m);   // §8(f)3, [12]
+kf_plan *plan_exact(kf_pipeline *p, const kf_model_params &m);   // §8(f)4, n <= 16
 kf_plan *plan_from_blocks(kf_pipeline *p, std::vector<std::vector<int>> blocks, bool check);
 bool dependence_legal(const kf_pipeline *p, const std::set<int> &P);
 bool header_legal(const kf_pipeline *p, const std::set<int> &P);
@@ -152,7 +154,7 @@ struct StreamInfo {
     std::map<int, Separable> sep; // local kernel -> factorisation
 };
 
-std::string kernel_name(int block);
+std::string kernel_name(const BlockInfo &b, int block);
 int env_int(const char *name, int dflt, int lo, int hi);
 StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b);
 std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block);

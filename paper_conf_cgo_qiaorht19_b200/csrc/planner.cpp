@@ -291,6 +291,139 @@ kf_plan *plan_fusion(kf_pipeline *p, const kf_model_params &m)
     return plan.release();
 }
 
+// ---------------------------------------------------------------------------
+// §8(f)3 -- the "basic" fusion of the authors' previous work [12], the paper's
+// comparison column: only point-to-point,
+// local-to-point and point-to-local fusion; a shared input (Fig. 2b) is
+// treated as an external dependence and rejected.  Reading R-18:
+// a block is basic-legal iff it is legal for Alg. 1 (dependence, resources,
+// header, profitability) AND it has exactly one source kernel, no kernel but
+// that source reads an image from outside the block, and no local kernel has
+// a local kernel upstream inside the block (that would be local-to-local).
+// [12] fuses pair-wise: edges are visited by decreasing benefit (ties: lower
+// producer, then lower consumer) and the two blocks an edge joins are merged
+// when the union is basic-legal, until a full pass merges nothing.
+static bool basic_legal(const kf_pipeline *p, const std::set<int> &P, const kf_model_params &m,
+                        const std::vector<EdgeInfo> &E)
+{
+    if (P.size() == 1) return true;
+    if (!is_legal(p, P, m, E)) return false;
+    auto pr = producers(p);
+    int nsrc = 0;
+    for (int k : P) {
+        bool has_prod = false;
+        for (int s : pr[k]) has_prod |= P.count(s) > 0;
+        if (has_prod) {
+            for (int img : p->ops[k].inputs)
+                if (!(img >= p->n_inputs && P.count(img - p->n_inputs))) return false;   // shared/external input
+        } else {
+            nsrc++;
+        }
+    }
+    if (nsrc != 1) return false;
+    for (int k : P) {
+        if (p->ops[k].kind != LOCAL) continue;
+        std::vector<int> st(pr[k].begin(), pr[k].end());   // walk the producers inside P
+        std::set<int> seen;
+        while (!st.empty()) {
+            int u = st.back();
+            st.pop_back();
+            if (!P.count(u) || !seen.insert(u).second) continue;
+            if (p->ops[u].kind == LOCAL) return false;   // local-to-local
+            for (int v : pr[u]) st.push_back(v);
+        }
+    }
+    return true;
+}
+
+kf_plan *plan_basic(kf_pipeline *p, const kf_model_params &m)
+{
+    if (p->ops.empty()) fail(KF_ERR_ARG, "pipeline has no kernels");
+    auto plan = std::make_unique<kf_plan>();
+    plan->edges = edge_weights(p, m);
+    const int n = (int)p->ops.size();
+    std::vector<int> lab(n);
+    for (int k = 0; k < n; k++) lab[k] = k;
+    std::vector<const EdgeInfo *> order;
+    for (const EdgeInfo &e : plan->edges)
+        if (e.profitable) order.push_back(&e);
+    std::stable_sort(order.begin(), order.end(), [](const EdgeInfo *a, const EdgeInfo *b) {
+        if (a->w != b->w) return a->w > b->w;
+        return a->ks != b->ks ? a->ks < b->ks : a->kd < b->kd;
+    });
+    for (bool changed = true; changed;) {
+        changed = false;
+        for (const EdgeInfo *e : order) {
+            const int a = lab[e->ks], b = lab[e->kd];
+            if (a == b) continue;
+            std::set<int> U;
+            for (int k = 0; k < n; k++)
+                if (lab[k] == a || lab[k] == b) U.insert(k);
+            if (!basic_legal(p, U, m, plan->edges)) continue;
+            for (int k = 0; k < n; k++)
+                if (lab[k] == b) lab[k] = a;
+            changed = true;
+        }
+    }
+    std::map<int, std::vector<int>> byl;
+    for (int k = 0; k < n; k++) byl[lab[k]].push_back(k);
+    for (auto &kv : byl) plan->blocks.push_back(kv.second);
+    finish_plan(p, plan.get());
+    return plan.release();
+}
+
+// ---------------------------------------------------------------------------
+// §8(f)4 -- exact planner: the maximum of Eq. 1 (sum of the weights of the
+// edges inside blocks, lexicographic (q, eps) as in Alg. 1) over ALL
+// partitions into legal blocks -- the exhaustive alternative the paper rules
+// out for large graphs (minimum-weight k-cut, NP-complete).
+// Subset DP, O(3^n): best(S) = max over legal B, min(S) in B, B subset of S,
+// of w(B) + best(S \ B).  Limited to n <= 16 kernels.  Ties keep the first
+// candidate in increasing sub-mask order (deterministic).
+kf_plan *plan_exact(kf_pipeline *p, const kf_model_params &m)
+{
+    const int n = (int)p->ops.size();
+    if (n == 0) fail(KF_ERR_ARG, "pipeline has no kernels");
+    if (n > 16) fail(KF_ERR_ARG, "exact planner is limited to 16 kernels (O(3^n))");
+    auto plan = std::make_unique<kf_plan>();
+    plan->edges = edge_weights(p, m);
+    const uint32_t full = (1u << n) - 1;
+    std::vector<char> legal(full + 1, 0);
+    std::vector<W2> w(full + 1);
+    for (uint32_t s = 1; s <= full; s++) {
+        std::set<int> S;
+        for (int k = 0; k < n; k++)
+            if (s >> k & 1) S.insert(k);
+        legal[s] = S.size() == 1 || is_legal(p, S, m, plan->edges);
+        if (!legal[s]) continue;
+        for (const EdgeInfo &e : plan->edges)
+            if ((s >> e.ks & 1) && (s >> e.kd & 1)) w[s] = w[s] + W2{e.q, e.eps};
+    }
+    std::vector<W2> best(full + 1);
+    std::vector<uint32_t> pick(full + 1, 0);
+    for (uint32_t s = 1; s <= full; s++) {
+        const uint32_t low = s & (~s + 1u), rest = s ^ low;
+        bool have = false;
+        // sub-masks B = low | r, r a sub-mask of rest, in increasing order
+        for (uint32_t r = 0;; r = (r - rest) & rest) {
+            const uint32_t B = low | r;
+            if (legal[B]) {
+                W2 c = w[B] + best[s ^ B];
+                if (!have || best[s] < c) { best[s] = c; pick[s] = B; have = true; }
+            }
+            if (r == rest) break;
+        }
+    }
+    for (uint32_t s = full; s; s ^= pick[s]) {
+        std::vector<int> b;
+        for (int k = 0; k < n; k++)
+            if (pick[s] >> k & 1) b.push_back(k);
+        plan->blocks.push_back(b);
+    }
+    finish_plan(p, plan.get());
+    return plan.release();
+}
+
 kf_plan *plan_from_blocks(kf_pipeline *p, std::vector<std::vector<int>> blocks, bool check)
 {
     auto plan = std::make_unique<kf_plan>();

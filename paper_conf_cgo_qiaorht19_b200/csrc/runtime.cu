@@ -165,22 +165,35 @@ struct CompiledBlock {
     }
 };
 
+constexpr int kHostBands = 8;   // kf_run_host pipeline depth (row bands)
+
 struct Runtime {
     std::map<uint64_t, std::shared_ptr<CompiledBlock>> modules;   // by source hash
     std::vector<void *> stage_in, stage_out;                      // kf_run_host staging
     size_t stage_bytes = 0;
     int device = -1;
+    // kf_run_host copy engines: H2D and D2H streams + per-band events
+    cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+    cudaEvent_t ev_in[kHostBands] = {}, ev_out[kHostBands] = {}, ev_start = nullptr, ev_done = nullptr;
     ~Runtime()
     {
         for (void *q : stage_in) cudaFree(q);
         for (void *q : stage_out) cudaFree(q);
+        for (int i = 0; i < kHostBands; i++) {
+            if (ev_in[i]) cudaEventDestroy(ev_in[i]);
+            if (ev_out[i]) cudaEventDestroy(ev_out[i]);
+        }
+        if (ev_start) cudaEventDestroy(ev_start);
+        if (ev_done) cudaEventDestroy(ev_done);
+        if (s_h2d) cudaStreamDestroy(s_h2d);
+        if (s_d2h) cudaStreamDestroy(s_d2h);
     }
 };
 
 // Compile-only path usable without a GPU (build() warms the in-tree cache).
 std::string compile_block_cubin(const kf_pipeline *p, const kf_plan *plan, int i)
 {
-    return compile_cubin(generate_block(p, plan->info[i], i), kernel_name(i));
+    return compile_cubin(generate_block(p, plan->info[i], i), kernel_name(plan->info[i], i));
 }
 
 void prepare(kf_pipeline *p, kf_plan *plan)
@@ -199,9 +212,9 @@ void prepare(kf_pipeline *p, kf_plan *plan)
         auto it = p->rt->modules.find(h);
         if (it == p->rt->modules.end()) {
             auto cb = std::make_shared<CompiledBlock>();
-            std::string cubin = compile_cubin(src, kernel_name((int)i));
+            std::string cubin = compile_cubin(src, kernel_name(plan->info[i], (int)i));
             cu_check(d.moduleLoadData(&cb->mod, cubin.data()), "cuModuleLoadData");
-            cu_check(d.moduleGetFunction(&cb->fn, cb->mod, kernel_name((int)i).c_str()), "cuModuleGetFunction");
+            cu_check(d.moduleGetFunction(&cb->fn, cb->mod, kernel_name(plan->info[i], (int)i).c_str()), "cuModuleGetFunction");
             cb->source = src;
             cb->si = stream_info(p, plan->info[i]);
             cu_check(d.occupancy(&cb->ctas_per_sm, cb->fn, kThreads, 0), "cuOccupancyMaxActiveBlocksPerMultiprocessor");
@@ -392,13 +405,20 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
     }
 }
 
+// End-to-end call with host buffers.  The image is cut into kHostBands row
+// bands and the three engines overlap: the H2D copy engine
+// uploads band k+1's input rows while the SMs compute band k (kf_run_band
+// semantics: border modes act at the global edges, so the result is identical
+// to one whole-image run) and the D2H engine downloads band k-1's output rows.
+// Band k waits only for the input rows it reads, [row0 - R, row1 + R).
+// REPEAT plans (no band mode) and tiny images run as one band.
 void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
               void *stream)
 {
     if (n_in != p->n_inputs || n_out != (int)p->outputs.size()) fail(KF_ERR_ARG, "wrong number of buffers");
     prepare(p, plan);
     Runtime &rt = *p->rt;
-    const size_t bytes = (size_t)p->W * p->H * 4;
+    const size_t row_bytes = (size_t)p->W * 4, bytes = row_bytes * p->H;
     if (rt.stage_bytes != bytes || rt.stage_in.size() != (size_t)n_in || rt.stage_out.size() != (size_t)n_out) {
         for (void *q : rt.stage_in) cudaFree(q);
         for (void *q : rt.stage_out) cudaFree(q);
@@ -410,11 +430,53 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
             if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
         rt.stage_bytes = bytes;
     }
+    if (!rt.s_h2d) {
+        KF_CUDA(cudaStreamCreateWithFlags(&rt.s_h2d, cudaStreamNonBlocking));
+        KF_CUDA(cudaStreamCreateWithFlags(&rt.s_d2h, cudaStreamNonBlocking));
+        for (int i = 0; i < kHostBands; i++) {
+            KF_CUDA(cudaEventCreateWithFlags(&rt.ev_in[i], cudaEventDisableTiming));
+            KF_CUDA(cudaEventCreateWithFlags(&rt.ev_out[i], cudaEventDisableTiming));
+        }
+        KF_CUDA(cudaEventCreateWithFlags(&rt.ev_start, cudaEventDisableTiming));
+        KF_CUDA(cudaEventCreateWithFlags(&rt.ev_done, cudaEventDisableTiming));
+    }
     cudaStream_t s = (cudaStream_t)stream;
-    for (int i = 0; i < n_in; i++) KF_CUDA(cudaMemcpyAsync(rt.stage_in[i], hin[i], bytes, cudaMemcpyHostToDevice, s));
+    bool repeat = false;
+    for (const auto &op : p->ops) repeat |= op.kind == LOCAL && op.mode == KF_REPEAT;
+    const int R = plan->halo_rows;
+    int nb = repeat ? 1 : std::max(1, std::min(kHostBands, p->H / std::max(64, 4 * R)));
     std::vector<const void *> din(rt.stage_in.begin(), rt.stage_in.end());
-    run(p, plan, din.data(), n_in, rt.stage_out.data(), n_out, stream, 0, p->H, 0, p->H);
-    for (int j = 0; j < n_out; j++) KF_CUDA(cudaMemcpyAsync(hout[j], rt.stage_out[j], bytes, cudaMemcpyDeviceToHost, s));
+    // the copy streams start after everything already queued on the caller's stream
+    KF_CUDA(cudaEventRecord(rt.ev_start, s));
+    KF_CUDA(cudaStreamWaitEvent(rt.s_h2d, rt.ev_start, 0));
+    KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_start, 0));
+    int copied = 0;   // input rows [0, copied) are queued on the H2D stream
+    for (int k = 0; k < nb; k++) {
+        const int r0 = (int)((long long)p->H * k / nb), r1 = (int)((long long)p->H * (k + 1) / nb);
+        const int need = k == nb - 1 ? p->H : std::min(p->H, r1 + R);
+        if (need > copied) {
+            for (int i = 0; i < n_in; i++)
+                KF_CUDA(cudaMemcpyAsync((char *)rt.stage_in[i] + copied * row_bytes,
+                                        (const char *)hin[i] + copied * row_bytes, (need - copied) * row_bytes,
+                                        cudaMemcpyHostToDevice, rt.s_h2d));
+            copied = need;
+        }
+        KF_CUDA(cudaEventRecord(rt.ev_in[k], rt.s_h2d));
+        KF_CUDA(cudaStreamWaitEvent(s, rt.ev_in[k], 0));
+        std::vector<void *> dout(n_out);
+        for (int j = 0; j < n_out; j++) dout[j] = nb == 1 ? rt.stage_out[j] : (char *)rt.stage_out[j] + r0 * row_bytes;
+        if (nb == 1)
+            run(p, plan, din.data(), n_in, dout.data(), n_out, stream, 0, p->H, 0, p->H);
+        else
+            run(p, plan, din.data(), n_in, dout.data(), n_out, stream, r0, r1, 0, p->H);
+        KF_CUDA(cudaEventRecord(rt.ev_out[k], s));
+        KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_out[k], 0));
+        for (int j = 0; j < n_out; j++)
+            KF_CUDA(cudaMemcpyAsync((char *)hout[j] + r0 * row_bytes, (const char *)rt.stage_out[j] + r0 * row_bytes,
+                                    (r1 - r0) * row_bytes, cudaMemcpyDeviceToHost, rt.s_d2h));
+    }
+    KF_CUDA(cudaEventRecord(rt.ev_done, rt.s_d2h));
+    KF_CUDA(cudaStreamWaitEvent(s, rt.ev_done, 0));
     KF_CUDA(cudaStreamSynchronize(s));
 }
 

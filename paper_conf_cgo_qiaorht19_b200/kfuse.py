@@ -64,6 +64,8 @@ _SIGS = {
                                   C.c_double, C.POINTER(KfInstr), C.c_int32, C.POINTER(KfCost), _I32P]),
     "kf_mark_output": (C.c_int, [_P, C.c_int32]),
     "kf_plan_fusion": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
+    "kf_plan_basic": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
+    "kf_plan_exact": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
     "kf_plan_unfused": (C.c_int, [_P, C.POINTER(_P)]),
     "kf_plan_from_blocks": (C.c_int, [_P, _I32P, C.POINTER(_P)]),
     "kf_plan_destroy": (None, [_P]),
@@ -195,6 +197,20 @@ class Pipeline:
         m = model_params(profile, **over) if isinstance(profile, str) else profile
         h = _P()
         _check(lib.kf_plan_fusion(self.h, C.byref(m), C.byref(h)))
+        return Plan(self, h)
+
+    def plan_basic(self, profile="paper", **over) -> "Plan":
+        """kf_plan_basic: the basic fusion of [12] (comparison column of Table I)."""
+        m = model_params(profile, **over) if isinstance(profile, str) else profile
+        h = _P()
+        _check(lib.kf_plan_basic(self.h, C.byref(m), C.byref(h)))
+        return Plan(self, h)
+
+    def plan_exact(self, profile="paper", **over) -> "Plan":
+        """kf_plan_exact: the optimum of Eq. 1 over all legal partitions (<= 16 kernels)."""
+        m = model_params(profile, **over) if isinstance(profile, str) else profile
+        h = _P()
+        _check(lib.kf_plan_exact(self.h, C.byref(m), C.byref(h)))
         return Plan(self, h)
 
     def plan_unfused(self) -> "Plan":

@@ -144,3 +144,73 @@ def test_generated_kernels_compile_for_sm100a(seed, tmp_path, monkeypatch):
     assert len(cubins) == len(plan.blocks)
     blob = cubins[0].read_bytes()
     assert blob[:4] == b"\x7fELF"
+
+
+# ----------------------------------------- basic [12] and exact planners (§8(f))
+
+
+@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10"])
+@pytest.mark.parametrize("profile", ["paper", "b200"])
+def test_basic_planner_matches_reference(wl, profile):
+    spec = P.WORKLOADS[wl](64, 64)
+    plan = K.Pipeline.from_spec(spec).plan_basic(profile)
+    assert plan.blocks == PL.basic_fusion(spec, _ref_model(profile))
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_basic_planner_matches_reference_on_random_dags(seed):
+    rng = random.Random(8000 + seed)
+    spec = P.random_pipeline(rng, 16, 16, rng.choice(["f32", "u8x4"]), rng.randint(1, 9))
+    profile = rng.choice(["paper", "b200"])
+    plan = K.Pipeline.from_spec(spec).plan_basic(profile)
+    assert plan.blocks == PL.basic_fusion(spec, _ref_model(profile))
+
+
+def _check_exact(spec, profile):
+    m = _ref_model(profile)
+    plan = K.Pipeline.from_spec(spec).plan_exact(profile)
+    best, _ = PL.brute_force(spec, m)
+    assert plan.objective == best
+    g = PL.graph(spec)
+    info = PL.edge_weights(g, m)
+    assert sorted(k for b in plan.blocks for k in b) == list(range(g.n))
+    for b in plan.blocks:
+        assert PL.is_legal(g, set(b), m, info)
+    assert K.Pipeline.from_spec(spec).plan_fusion(profile).objective <= plan.objective
+    return plan
+
+
+@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10"])
+@pytest.mark.parametrize("profile", ["paper", "b200"])
+def test_exact_planner_equals_bruteforce_on_workloads(wl, profile):
+    _check_exact(P.WORKLOADS[wl](64, 64), profile)
+
+
+@pytest.mark.parametrize("seed", range(50))
+def test_exact_planner_equals_bruteforce_on_random_dags(seed):
+    rng = random.Random(9000 + seed)
+    spec = P.random_pipeline(rng, 16, 16, rng.choice(["f32", "u8x4"]), rng.randint(1, 8))
+    _check_exact(spec, rng.choice(["paper", "b200"]))
+
+
+def test_exact_planner_beats_min_cut_counterexample():
+    """Alg. 1 reaches 350 on the 5-local chain, the optimum is 550."""
+    p = P.Pipeline("chain", 32, 32, "f32")
+    x = p.input()
+    for k, n_alu in enumerate([12, 8, 4, 2, 1]):
+        x = p.local(f"l{k}", x, [[1] * 3] * 3, "clamp", cost=(n_alu, 0))
+    p.output(x)
+    over = dict(ts=1.0, c_alu=1.0, c_mshared=2.0)
+    pipe = K.Pipeline.from_spec(p.spec())
+    assert pipe.plan_fusion("paper", **over).objective == (350 << 20, 0)
+    assert K.Pipeline.from_spec(p.spec()).plan_exact("paper", **over).objective == (550 << 20, 0)
+
+
+def test_exact_planner_size_limit():
+    p = P.Pipeline("long", 16, 16, "f32")
+    x = p.input()
+    for k in range(17):
+        x = p.point(f"p{k}", [x], [("LOAD", 0, 0), ("CONST", 0, 1.0), ("ADD", 0, 0)])
+    p.output(x)
+    with pytest.raises(K.KfError):
+        K.Pipeline.from_spec(p.spec()).plan_exact("paper")

@@ -169,14 +169,40 @@ def test_full_size_sampled(cfg):
 
 # ---------------------------------------------------------- other entry points
 
-def test_run_host_equals_run():
-    spec = P.harris(300, 200)
+@pytest.mark.parametrize("wl", ["harris", "deep10", "unsharp"])
+@pytest.mark.parametrize("kind", ["unfused", "paper", "b200"])
+@pytest.mark.parametrize("size", [(300, 200), (64, 1030), (40, 9)])
+def test_run_host_equals_run(wl, kind, size):
+    """kf_run_host (row-band pipelined H2D / compute / D2H) == kf_run, bit for bit."""
+    spec = P.WORKLOADS[wl](*size)
     ins = _inputs(spec, 4)
-    plan = make_plan(spec, "b200")
+    plan = make_plan(spec, kind)
     dev = run_gpu(spec, plan, ins)[0]
     out = np.empty_like(dev)
-    plan.run_host([np.ascontiguousarray(ins[0])], [out])
+    plan.run_host([np.ascontiguousarray(a) for a in ins], [out])
     np.testing.assert_array_equal(out, dev)
+
+
+def test_run_host_repeat_and_pinned():
+    """REPEAT plans (one band) and pinned host buffers on a non-default stream."""
+    spec = P.harris(256, 300, "repeat")
+    ins = _inputs(spec, 5)
+    plan = make_plan(spec, "b200")
+    dev = run_gpu(spec, plan, ins)[0]
+    hin = torch.from_numpy(np.ascontiguousarray(ins[0])).pin_memory()
+    hout = torch.empty(dev.shape, dtype=torch.float32).pin_memory()
+    s = torch.cuda.Stream()
+    plan.run_host([hin], [hout], s)
+    np.testing.assert_array_equal(hout.numpy(), dev)
+    spec = P.harris(256, 1024)
+    ins = _inputs(spec, 6)
+    plan = make_plan(spec, "b200")
+    dev = run_gpu(spec, plan, ins)[0]
+    hin = torch.from_numpy(np.ascontiguousarray(ins[0])).pin_memory()
+    hout = torch.empty(dev.shape, dtype=torch.float32).pin_memory()
+    for _ in range(3):   # repeated calls reuse the staging buffers, streams and events
+        plan.run_host([hin], [hout], s)
+    np.testing.assert_array_equal(hout.numpy(), dev)
 
 
 @pytest.mark.parametrize("wl", ["harris", "deep10", "unsharp"])

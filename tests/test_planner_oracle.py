@@ -239,3 +239,70 @@ def test_deep10_reaches_bruteforce_optimum():
     for m in (PL.PAPER_PROFILE, PL.B200_PROFILE):
         got, best = PL.get_legal_partitions(s, m).beta, PL.brute_force(s, m)[0]
         assert got[0] == best[0] and got <= best
+
+
+# ------------------------------------------------ basic fusion [12] (§8(f)3)
+
+
+@pytest.mark.parametrize("prof", [PL.PAPER_PROFILE, PL.B200_PROFILE])
+def test_basic_fusion_paper_statements(prof):
+    """PAPER.md:1414-1425 (Table I discussion): the basic fusion of [12] gains most
+    on Enhance (a local and two point operators, fully fused); it "failed in
+    optimizing" Sobel (local-to-local) and Unsharp (shared input); on Harris and
+    ShiTomasi it detects the point-to-local scenarios (the three square ->
+    Gaussian pairs of Fig. 3)."""
+    e = P.enhance(64, 64)
+    assert PL.basic_fusion(e, prof) == [list(range(len(e["ops"])))]
+    for wl in ("sobel", "unsharp"):
+        s = P.WORKLOADS[wl](64, 64)
+        assert PL.basic_fusion(s, prof) == [[k] for k in range(len(s["ops"]))]
+    for wl in ("harris", "shitomasi"):
+        s = P.WORKLOADS[wl](64, 64)
+        multi = [names(s, b) for b in PL.basic_fusion(s, prof) if len(b) > 1]
+        assert sorted(multi) == [["sx", "gx"], ["sxy", "gxy"], ["sy", "gy"]]
+
+
+def test_basic_rules_negative_controls():
+    """Hand-built two-kernel blocks: point-to-local and local-to-point are basic-legal,
+    local-to-local and a shared input are not."""
+    p = P.Pipeline("ctl", 32, 32, "f32")
+    x = p.input()
+    a = p.point("a", [x], [("LOAD", 0, 0), ("CONST", 0, 2.0), ("MUL", 0, 0)])
+    b = p.local("b", a, [[1, 2, 1], [2, 4, 2], [1, 2, 1]], "clamp")
+    c = p.local("c", b, [[1, 2, 1], [2, 4, 2], [1, 2, 1]], "clamp")
+    d = p.point("d", [c, x], [("LOAD", 0, 0), ("LOAD", 1, 0), ("ADD", 0, 0)])
+    p.output(d)
+    s = p.spec()
+    g = PL.graph(s)
+    m = PL.Model(c_mshared=5.0, phi_mode=1)
+    info = PL.edge_weights(g, m)
+    assert PL.is_legal(g, {0, 1}, m, info) and PL.basic_legal(g, {0, 1}, m, info)        # point-to-local
+    assert PL.is_legal(g, {1, 2}, m, info) and not PL.basic_legal(g, {1, 2}, m, info)    # local-to-local
+    assert not PL.is_legal(g, {2, 3}, m, info)          # d reads x, the source c does not: Fig. 2d
+    assert not PL.basic_legal(g, {0, 1, 2}, m, info)   # local-to-local behind a point
+    q = P.Pipeline("shared", 32, 32, "f32")            # Fig. 2b: the shared input
+    x = q.input()
+    a = q.point("a", [x], [("LOAD", 0, 0), ("CONST", 0, 2.0), ("MUL", 0, 0)])
+    e = q.point("e", [a, x], [("LOAD", 0, 0), ("LOAD", 1, 0), ("SUB", 0, 0)])
+    q.output(e)
+    g = PL.graph(q.spec())
+    info = PL.edge_weights(g, m)
+    assert PL.is_legal(g, {0, 1}, m, info) and not PL.basic_legal(g, {0, 1}, m, info)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_basic_fusion_is_legal_cover_below_optimum(seed):
+    """Every basic block is basic-legal (hence IsLegal), the blocks partition the
+    kernels, and beta_basic <= beta* (the exhaustive optimum)."""
+    rng = random.Random(7000 + seed)
+    s = P.random_pipeline(rng, 16, 16, rng.choice(["f32", "u8x4"]), rng.randint(2, 7))
+    m = rng.choice([PL.PAPER_PROFILE, PL.B200_PROFILE])
+    blocks = PL.basic_fusion(s, m)
+    g = PL.graph(s)
+    info = PL.edge_weights(g, m)
+    assert sorted(k for b in blocks for k in b) == list(range(g.n))
+    beta = (0, 0)
+    for b in blocks:
+        assert PL.basic_legal(g, set(b), m, info)
+        beta = PL._add(beta, PL.block_weight(set(b), info))
+    assert beta <= PL.brute_force(s, m)[0]
