@@ -35,10 +35,13 @@ UNIT = "Mpixel/s"
 DATA = "synthetic: counter-based SplitMix64 uniform [0,1) images (kf_inputs/gen.py), as the paper's random images"
 # algorithmic DRAM bytes per pixel of each plan: every launched kernel
 # reads its external inputs once and writes its output once (f32: 4 B per image)
-ALG_BYTES = {"harris": {"unfused": 84, "paper": 60, "b200": 8},
-             "shitomasi": {"unfused": 84, "paper": 60, "b200": 8},
-             "unsharp": {"unfused": 44, "paper": 8, "b200": 8},
-             "deep10": {"unfused": 100, "paper": 92, "b200": 8}}
+ALG_BYTES = {"harris": {"unfused": 84, "basic": 60, "paper": 60, "b200": 8},
+             "shitomasi": {"unfused": 84, "basic": 60, "paper": 60, "b200": 8},
+             "unsharp": {"unfused": 44, "basic": 44, "paper": 8, "b200": 8},
+             "deep10": {"unfused": 100, "basic": 92, "paper": 92, "b200": 8}}
+PLANS = ("unfused", "basic", "paper", "b200")
+# the other BASELINE.json configs, timed beside the headline (parity cases otherwise)
+EXTRA_CONFIGS = ("C1", "C2", "C3s", "C4")
 
 
 def load_peaks() -> dict:
@@ -49,6 +52,24 @@ def load_peaks() -> dict:
         return {"hbm_gbs": float(d["hbm_gbs"]), "source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
     except Exception:
         return {"hbm_gbs": 6650.0, "source": "fallback 6.65 TB/s (B200_PROFILING.md)"}
+
+
+def ncu_inst(cfg: str, plan: str):
+    """warp instructions per pixel of the fused kernel from a committed ncu capture, if any."""
+    path = os.path.join(ROOT, "profiles", "ncu_inst.json")
+    try:
+        with open(path) as f:
+            return json.load(f).get(f"{cfg}:{plan}")
+    except Exception:
+        return None
+
+
+def make_plan(p, kind):
+    if kind == "unfused":
+        return p.plan_unfused()
+    if kind == "basic":
+        return p.plan_basic("paper")
+    return p.plan_fusion(kind)
 
 
 def ncu_traffic(cfg: str, plan: str):
@@ -212,13 +233,13 @@ def bench_single(args, cfg_name, spec, seed) -> None:
     stream = torch.cuda.Stream()
     results = {}
     plans = {}
-    for kind in ("unfused", "paper", "b200"):
+    for kind in PLANS:
         p = K.Pipeline.from_spec(spec)
-        plan = p.plan_unfused() if kind == "unfused" else p.plan_fusion(kind)
+        plan = make_plan(p, kind)
         plan.prepare()
         plans[kind] = (p, plan)
     # headline plan last, with clocks sampled during its timed region
-    order = [k for k in ("unfused", "paper", "b200") if k != args.plan] + [args.plan]
+    order = [k for k in PLANS if k != args.plan] + [args.plan]
     clocks = None
     for kind in order:
         p, plan = plans[kind]
@@ -263,6 +284,8 @@ def bench_single(args, cfg_name, spec, seed) -> None:
         dt, n = cpu_oracle_run(spec["name"], W, H if spec["dtype"] == "f32" else 256, seed)
         cpu = {"value": round(n / dt / 1e6, 3), "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": f"one {W}x{H if spec['dtype'] == 'f32' else 256} image of the workload, unfused fp64 oracle, 1 thread"}
+    del ins, outs
+    extra = {} if args.no_extra else bench_extra(args, stream, torch, clocks)
     out = {
         "metric": METRIC, "value": head["mpix_s"], "unit": UNIT, "n_gpus": 1, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": head["ms_per_step"], "higher_is_better": True, "scaling": "weak",
@@ -272,8 +295,58 @@ def bench_single(args, cfg_name, spec, seed) -> None:
         "gpu_launches": args.steps * hplan.num_launches, "clocks": clocks,
         "plans": results,
         "fused_vs_unfused": round(results["unfused"]["ms_per_step"] / head["ms_per_step"], 3),
+        "workloads": extra,
     }
     print(json.dumps(out))
+
+
+def bench_extra(args, stream, torch, clocks) -> dict:
+    """The other BASELINE.json configs (C1 Harris 256^2, C2 Unsharp 2048^2, C3s
+    ShiTomasi 4096^2, C4 deep10 7680x4320 u8x4), every plan, timed like the
+    headline (CUDA-graph replay, rotating buffer sets larger than L2).  The fused
+    plan gets its HBM fraction (algorithmic bytes) and, where a committed ncu
+    capture gives its instruction count, its issue fraction (C4 is ALU-bound,
+    SURVEY §8(d)): warp instructions / (148 SMs x 4 schedulers x SM clock)."""
+    from kf_inputs import gen
+    from kf_inputs import pipelines as P
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+    peaks = load_peaks()
+    sm_hz = ((clocks or {}).get("sm_mhz") or 1965.0) * 1e6
+    n_sm = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+    res = {}
+    for cfg in EXTRA_CONFIGS:
+        spec, seed = P.config(cfg)
+        W, H = spec["width"], spec["height"]
+        px = W * H
+        host = gen.image(spec["dtype"], seed, W, H)
+        tdt = torch.float32 if spec["dtype"] == "f32" else torch.uint8
+        oshape = (H, W) if spec["dtype"] == "f32" else (H, W, 4)
+        nsets = max(2, min(8, int(512e6 // (8 * px))))     # sets x (in + out) >= ~512 MB > L2 where possible
+        ins = [torch.from_numpy(host).cuda() for _ in range(nsets)]
+        outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(nsets)]
+        d = {"workload": f"{spec['name']} {W}x{H} {spec['dtype']}", "plans": {}}
+        for kind in PLANS:
+            p = K.Pipeline.from_spec(spec)
+            plan = make_plan(p, kind)
+            plan.prepare()
+            steps = 20 if px > 2e7 else 100
+            ms = time_plan(plan, ins, outs, steps, 3, stream, torch)
+            ab = ALG_BYTES.get(spec["name"], {}).get(kind)
+            d["plans"][kind] = {"ms_per_step": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
+                                "launches": plan.num_launches, "alg_bytes_per_px": ab,
+                                "hbm_frac": round(ab * px / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4) if ab else None}
+        f = d["plans"]["b200"]
+        d["fused_vs_unfused"] = round(d["plans"]["unfused"]["ms_per_step"] / f["ms_per_step"], 3)
+        ipp = ncu_inst(cfg, "b200")
+        if ipp:
+            issue = ipp * px / (f["ms_per_step"] * 1e-3)
+            d["issue"] = {"bound": "alu", "warp_inst_per_px": ipp, "achieved": round(issue / 1e9, 1),
+                          "peak": round(n_sm * 4 * sm_hz / 1e9, 1), "unit": "G warp-inst/s",
+                          "frac": round(issue / (n_sm * 4 * sm_hz), 4),
+                          "source": "profiles/ncu_inst.json (ncu smsp__inst_executed.sum / px)"}
+        res[cfg] = d
+        del ins, outs
+    return res
 
 
 def bench_multi(args, cfg_name, spec, seed) -> None:
@@ -293,7 +366,7 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     Htot = Hb * world                                 # weak scaling: one band per GPU
     gspec = P.WORKLOADS[spec["name"]](W, Htot)
     p = K.Pipeline.from_spec(gspec)
-    plan = p.plan_unfused() if args.plan == "unfused" else p.plan_fusion(args.plan)
+    plan = make_plan(p, args.plan)
     plan.prepare()
     band = KD.partition(Htot, world, rank, plan.halo_rows)
     host = gen.image(gspec["dtype"], seed, W, Htot, band.in0, band.in1)
@@ -304,9 +377,10 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(nsets)]
     stream = torch.cuda.current_stream()
 
-    def step(i):
-        KD.exchange_halos(ins[i % nsets], band)
-        KD.run_band(plan, band, [ins[i % nsets]], [outs[i % nsets]], stream)
+    side = torch.cuda.Stream()
+
+    def step(i):   # halo exchange (NCCL) overlapped with the band's core rows
+        KD.run_step_overlapped(plan, band, [ins[i % nsets]], [outs[i % nsets]], side)
 
     for i in range(args.warmup):
         step(i)
@@ -333,7 +407,7 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": DATA,
             "config": config_dict(cfg_name, gspec, args.plan,
-                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows via NCCL send/recv",
+                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows via NCCL send/recv overlapped with the core rows",
                                    "band": f"{Hb}x{W} per GPU"}),
             "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": round(ach / peaks["hbm_gbs"], 4), "traffic": None,
@@ -352,8 +426,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="kfuse", choices=["kfuse", "reference"])
     ap.add_argument("--config", default="C3")
-    ap.add_argument("--plan", default="b200", choices=["b200", "paper", "unfused"])
+    ap.add_argument("--plan", default="b200", choices=list(PLANS))
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-extra", action="store_true", help="skip the other BASELINE configs")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     from kf_inputs import pipelines as P

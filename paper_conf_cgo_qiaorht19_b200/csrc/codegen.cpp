@@ -25,6 +25,7 @@
 //   * blocks whose local kernels all use REPEAT use a torus slot model in the
 //     frame: slot p holds the value at p mod n (wrap needs no exchange).
 #include <algorithm>
+#include <climits>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -197,6 +198,284 @@ struct ProgEmitter {
         return ev(st.back());
     }
 };
+
+// ======================================================================= SWAR
+// u8x4 pipelines in the interior path: two channels per 32-bit register, one
+// per 16-bit lane ("SWAR").  A pixel is two registers, lo =
+// (c0, c1) and hi = (c2, c3).  A value of the method (an integer per channel,
+// int32 semantics, R-16) is held with a compile-time bias B >= 0 in every lane
+// (lane = v + B) and a compile-time interval [vlo, vhi] of v, the same for all
+// channels.  Interval analysis at code-generation time decides whether a
+// kernel fits: every materialised lane must stay in [0, 65535].
+//   * linear forms sum c_i x_i + k (ADD/SUB/NEG/SHL/MUL-by-constant and every
+//     mask accumulation) are evaluated with plain 32-bit integer arithmetic on
+//     both registers: arithmetic mod 2^32 is a ring, so whenever the final
+//     lanes are in range the packed result is exact, whatever the order or the
+//     intermediate wrap-arounds (IADD3 / LEA / IMAD serve two channels each);
+//   * SHR n (arithmetic, floor): bias aligned to 2^n, then (x >> n) & mask;
+//   * MIN / MAX / CLAMP / SAT: VIMNMX.U16x2 on equal biases;
+//   * everything else (DIV, ABS, SELECT, LUT, variable products, overflowing
+//     ranges) makes the kernel fall back to per-channel int32 (I4) code.
+// Kernel outputs are saturated to [0, 255] (R-16), normalised to bias 0 and
+// packed to uchar4 with one PRMT; ring rows are unpacked with two.
+struct SwReg {
+    std::string lo, hi;
+    long long B = 0, vlo = 0, vhi = 255;
+};
+struct SwLin {
+    std::vector<std::pair<long long, SwReg>> t;
+    long long k = 0;
+};
+struct SwFail {};
+
+static long long floordiv(long long a, long long b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
+
+struct SwEmitter {
+    std::ostringstream *o = nullptr;   // null: interval-only dry run (feasibility)
+    int *tmp = nullptr;
+    std::string ind;
+    std::string var() { return "w" + std::to_string((*tmp)++); }
+    static std::string lit(long long v)   // v * 0x10001 as an unsigned literal (mod 2^32)
+    {
+        const unsigned long long u = (unsigned long long)(v * 65537LL) & 0xffffffffULL;
+        char b[32];
+        std::snprintf(b, sizeof b, "0x%llxu", u);
+        return b;
+    }
+    static SwLin of(const SwReg &r) { return SwLin{{{1, r}}, 0}; }
+    static SwLin cst(long long k) { return SwLin{{}, k}; }
+    static SwLin add(SwLin a, const SwLin &b, long long sb = 1)
+    {
+        for (auto &t : b.t) a.t.push_back({sb * t.first, t.second});
+        a.k += sb * b.k;
+        return a;
+    }
+    static SwLin scale(SwLin a, long long c)
+    {
+        for (auto &t : a.t) t.first *= c;
+        a.k *= c;
+        return a;
+    }
+    static void interval(const SwLin &l, long long &lo, long long &hi)
+    {
+        lo = hi = l.k;
+        for (auto &t : l.t) {
+            const long long a = t.first * t.second.vlo, b = t.first * t.second.vhi;
+            lo += std::min(a, b);
+            hi += std::max(a, b);
+        }
+    }
+    // materialise with a bias >= minB, multiple of `align`
+    SwReg mat(const SwLin &l, long long align = 1, long long minB = 0)
+    {
+        long long lo, hi;
+        interval(l, lo, hi);
+        long long B = std::max(std::max(0LL, -lo), minB);
+        B = (B + align - 1) / align * align;
+        if (hi + B > 65535 || lo + B < 0) throw SwFail{};
+        if (l.t.size() == 1 && l.t[0].first == 1 && l.k == 0 && l.t[0].second.B == B) return l.t[0].second;
+        long long K = B + l.k;
+        for (auto &t : l.t) {
+            if (std::llabs(t.first) > 65535) throw SwFail{};
+            K -= t.first * t.second.B;
+        }
+        SwReg r;
+        r.B = B;
+        r.vlo = lo;
+        r.vhi = hi;
+        if (o) {
+            r.lo = var();
+            r.hi = var();
+            for (int h = 0; h < 2; h++) {
+                std::string e;
+                for (auto &t : l.t) {
+                    const std::string &x = h ? t.second.hi : t.second.lo;
+                    const long long c = t.first;
+                    if (c == 0) continue;
+                    if (c == 1) e += (e.empty() ? "" : " + ") + x;
+                    else if (c == -1) e += (e.empty() ? "0u - " : " - ") + x;
+                    else if (c > 0) e += (e.empty() ? "" : " + ") + std::to_string(c) + "u * " + x;
+                    else e += (e.empty() ? "0u - " : " - ") + std::to_string(-c) + "u * " + x;
+                }
+                e += (e.empty() ? "" : " + ") + lit(K);
+                *o << ind << "const unsigned " << (h ? r.hi : r.lo) << " = " << e << ";\n";
+            }
+        }
+        return r;
+    }
+    SwReg shr(const SwReg &x, int n)
+    {
+        if (n <= 0) return x;
+        if (n >= 16) throw SwFail{};
+        SwReg a = mat(of(x), 1LL << n);
+        SwReg r;
+        r.B = a.B >> n;
+        r.vlo = floordiv(a.vlo, 1LL << n);
+        r.vhi = floordiv(a.vhi, 1LL << n);
+        if (o) {
+            r.lo = var();
+            r.hi = var();
+            const std::string m = lit(0xffff >> n);
+            *o << ind << "const unsigned " << r.lo << " = (" << a.lo << " >> " << n << ") & " << m << ";\n";
+            *o << ind << "const unsigned " << r.hi << " = (" << a.hi << " >> " << n << ") & " << m << ";\n";
+        }
+        return r;
+    }
+    SwReg minmax(const SwReg &a0, const SwReg &b0, bool mx)
+    {
+        const long long B = std::max(a0.B, b0.B);
+        SwReg a = mat(of(a0), 1, B), b = mat(of(b0), 1, B);
+        if (a.B != b.B) throw SwFail{};
+        SwReg r;
+        r.B = a.B;
+        r.vlo = mx ? std::max(a.vlo, b.vlo) : std::min(a.vlo, b.vlo);
+        r.vhi = mx ? std::max(a.vhi, b.vhi) : std::min(a.vhi, b.vhi);
+        if (o) {
+            r.lo = var();
+            r.hi = var();
+            const char *fn = mx ? "__vmaxu2" : "__vminu2";
+            *o << ind << "const unsigned " << r.lo << " = " << fn << "(" << a.lo << ", " << b.lo << ");\n";
+            *o << ind << "const unsigned " << r.hi << " = " << fn << "(" << a.hi << ", " << b.hi << ");\n";
+        }
+        return r;
+    }
+    SwReg clamp(const SwReg &x0, long long lo, long long hi)
+    {
+        SwReg x = x0;
+        if (lo > hi) throw SwFail{};
+        if (x.vhi <= lo) return mat(cst(lo));   // constant results
+        if (x.vlo >= hi) return mat(cst(hi));
+        if (x.vlo < lo) {
+            SwReg r = x;
+            r.vlo = lo;
+            if (o) {
+                r.lo = var();
+                r.hi = var();
+                *o << ind << "const unsigned " << r.lo << " = __vmaxu2(" << x.lo << ", " << lit(lo + x.B) << ");\n";
+                *o << ind << "const unsigned " << r.hi << " = __vmaxu2(" << x.hi << ", " << lit(lo + x.B) << ");\n";
+            }
+            x = r;
+        }
+        if (x.vhi > hi) {
+            SwReg r = x;
+            r.vhi = hi;
+            r.vlo = std::min(x.vlo, hi);
+            if (o) {
+                r.lo = var();
+                r.hi = var();
+                *o << ind << "const unsigned " << r.lo << " = __vminu2(" << x.lo << ", " << lit(hi + x.B) << ");\n";
+                *o << ind << "const unsigned " << r.hi << " = __vminu2(" << x.hi << ", " << lit(hi + x.B) << ");\n";
+            }
+            x = r;
+        }
+        return x;
+    }
+    // kernel boundary: saturate to [0, 255] and normalise to bias 0 (R-16)
+    SwReg sat_norm(const SwLin &l) { return mat(of(clamp(mat(l), 0, 255))); }
+    SwReg unpack(const std::string &u)
+    {
+        SwReg r;
+        if (o) {
+            r.lo = var();
+            r.hi = var();
+            *o << ind << "const unsigned " << r.lo << " = __byte_perm(" << u << ", 0u, 0x4140);\n";
+            *o << ind << "const unsigned " << r.hi << " = __byte_perm(" << u << ", 0u, 0x4342);\n";
+        }
+        return r;
+    }
+    std::string pack(const SwReg &x)   // requires bias 0 and [0, 255]
+    {
+        if (x.B != 0 || x.vlo < 0 || x.vhi > 255) throw SwFail{};
+        return "__byte_perm(" + x.lo + ", " + x.hi + ", 0x6420)";
+    }
+    // postfix op-IR over linear forms (LOAD k = loads[k]; a local op's post: LOAD 0 = acc)
+    SwLin prog(const Op &op, const std::vector<SwLin> &loads)
+    {
+        std::vector<SwLin> st;
+        auto pop = [&] { SwLin v = st.back(); st.pop_back(); return v; };
+        auto isc = [](const SwLin &l) { return l.t.empty(); };
+        for (const Instr &in : op.prog) {
+            switch (in.op) {
+            case KF_OP_LOAD: st.push_back(loads[op.kind == LOCAL ? 0 : in.arg]); break;
+            case KF_OP_CONST: {
+                const double c = in.imm;
+                if (c != std::floor(c) || std::fabs(c) > 65535) throw SwFail{};
+                st.push_back(cst((long long)c));
+                break;
+            }
+            case KF_OP_ADD: { SwLin b = pop(), a = pop(); st.push_back(add(a, b)); break; }
+            case KF_OP_SUB: { SwLin b = pop(), a = pop(); st.push_back(add(a, b, -1)); break; }
+            case KF_OP_NEG: st.push_back(scale(pop(), -1)); break;
+            case KF_OP_MUL: {
+                SwLin b = pop(), a = pop();
+                if (isc(b)) st.push_back(scale(a, b.k));
+                else if (isc(a)) st.push_back(scale(b, a.k));
+                else throw SwFail{};
+                break;
+            }
+            case KF_OP_SHL:
+                if (in.arg < 0 || in.arg > 15) throw SwFail{};
+                st.push_back(scale(pop(), 1LL << in.arg));
+                break;
+            case KF_OP_SHR: {
+                SwLin a = pop();
+                if (isc(a)) { st.push_back(cst(a.k >> in.arg)); break; }
+                st.push_back(of(shr(mat(a), in.arg)));
+                break;
+            }
+            case KF_OP_MIN: case KF_OP_MAX: {
+                SwLin b = pop(), a = pop();
+                const bool mx = in.op == KF_OP_MAX;
+                if (isc(a) && isc(b)) st.push_back(cst(mx ? std::max(a.k, b.k) : std::min(a.k, b.k)));
+                else if (isc(b)) st.push_back(of(mx ? clamp(mat(a), b.k, LLONG_MAX / 4) : clamp(mat(a), LLONG_MIN / 4, b.k)));
+                else if (isc(a)) st.push_back(of(mx ? clamp(mat(b), a.k, LLONG_MAX / 4) : clamp(mat(b), LLONG_MIN / 4, a.k)));
+                else st.push_back(of(minmax(mat(a), mat(b), mx)));
+                break;
+            }
+            case KF_OP_CLAMP: {
+                SwLin hi = pop(), lo = pop(), x = pop();
+                if (!isc(lo) || !isc(hi)) throw SwFail{};
+                st.push_back(of(clamp(mat(x), lo.k, hi.k)));
+                break;
+            }
+            case KF_OP_SAT_U8: st.push_back(of(clamp(mat(pop()), 0, 255))); break;
+            default: throw SwFail{};   // DIV, ABS, SELECT_GT, LUT, POW, ...
+            }
+        }
+        return st.back();
+    }
+};
+
+// Can kernel k run in SWAR form?  Interval-only dry run of the same emitter
+// (its inputs are kernel outputs or input images: always [0, 255]).
+static bool swar_feasible(const Op &op, const Separable &sp)
+{
+    int tmp = 0;
+    SwEmitter e;
+    e.tmp = &tmp;
+    try {
+        SwReg x;   // a [0, 255] value
+        SwLin acc;
+        if (op.kind == POINT) {
+            std::vector<SwLin> loads(op.inputs.size(), SwEmitter::of(x));
+            e.clamp(e.mat(e.prog(op, loads)), 0, 255);
+            return true;
+        }
+        if (sp.ok) {
+            SwLin v;
+            for (double c : sp.col) if (c != 0.0) v = SwEmitter::add(v, SwEmitter::scale(SwEmitter::of(x), (long long)c));
+            SwReg vr = e.mat(v);
+            for (double c : sp.row) if (c != 0.0) acc = SwEmitter::add(acc, SwEmitter::scale(SwEmitter::of(vr), (long long)c));
+        } else {
+            for (double m : op.mask) if (m != 0.0) acc = SwEmitter::add(acc, SwEmitter::scale(SwEmitter::of(x), (long long)m));
+        }
+        SwLin r = op.prog.empty() ? acc : e.prog(op, {acc});
+        e.clamp(e.mat(r), 0, 255);
+        return true;
+    } catch (const SwFail &) {
+        return false;
+    }
+}
 
 // ====================================================================== frame
 // Slow path: 2-D tiles with shared-memory staging and index exchange.  Used
@@ -442,6 +721,8 @@ struct StreamGen {
     // per-iteration memo: (image, ring slot, column) -> unpacked value variable
     std::map<std::tuple<int, int, int>, std::string> val_memo;
     std::map<std::tuple<std::string, int, int>, std::string> shfl_memo;   // (var, lane offset, edge key)
+    std::map<std::tuple<int, int, int>, SwReg> sw_memo;                     // SWAR values (image, slot, column)
+    std::map<std::tuple<std::string, int, int>, SwReg> swsh_memo;          // SWAR shuffles
     // variant being emitted
     int dir = 1;
     bool el = false, er = false;
@@ -615,8 +896,7 @@ struct StreamGen {
     // compile-time constant u of a peeled edge iteration (rows relative to the
     // strip start = the image edge), so taps outside the image are remapped;
     // u < 0: steady state, no remap.  Returns an empty vector for a constant row.
-    std::vector<std::string> tap_row(int kimg, const Op &op, int in, int dyp, int j, int u, bool &is_const,
-                                     const std::string &ind)
+    int tap_slot(int kimg, const Op &op, int in, int dyp, int j, int u, bool &is_const) const
     {
         const int L = si.L;
         int s = sl(in, HY(kimg) - HY(in) + dyp, j);
@@ -628,11 +908,18 @@ struct StreamGen {
                 const int m = edge_map(op.mode, rr);
                 if (m < 0) {
                     is_const = true;
-                    return {};
+                    return -1;
                 }
                 s = sl(in, m + 2 * L - HY(in) - u, j);   // the iteration that computed row m of `in`
             }
         }
+        return s;
+    }
+    std::vector<std::string> tap_row(int kimg, const Op &op, int in, int dyp, int j, int u, bool &is_const,
+                                     const std::string &ind)
+    {
+        const int s = tap_slot(kimg, op, in, dyp, j, u, is_const);
+        if (is_const) return {};
         last_slot = s;
         std::vector<std::string> row;
         for (int v = 0; v < V; v++) row.push_back(value(in, s, v, ind));
@@ -640,10 +927,140 @@ struct StreamGen {
     }
     int last_slot = 0;   // ring slot of the last tap_row (pair access in pair mode)
 
+    // ---- SWAR form of u8x4 kernels
+    SwEmitter swe(const std::string &ind) { SwEmitter e; e.o = &o; e.tmp = &tmp; e.ind = ind; return e; }
+    // value of image img at ring slot s, column v (bias 0, [0, 255]): memo or unpack
+    SwReg svalue(int img, int s, int v, const std::string &ind)
+    {
+        auto key = std::make_tuple(img, s, v);
+        auto it = sw_memo.find(key);
+        if (it != sw_memo.end()) return it->second;
+        SwReg r = swe(ind).unpack(ring(img, s, v));
+        sw_memo[key] = r;
+        return r;
+    }
+    // SWAR twin of at_col: own register or warp shuffle (both halves); in an
+    // edge chunk the edge lane substitutes its border-mapped own register or,
+    // for CONSTANT, `csub` (a value with the row's bias)
+    SwReg at_col_sw(const std::vector<SwReg> &row, int q, const Op &op, long long csub, const std::string &ind)
+    {
+        if (q >= 0 && q < V) return row[q];
+        int lo = q >= 0 ? q / V : -((-q + V - 1) / V);
+        int idx = q - lo * V;
+        const bool edge = (q < 0 && el) || (q >= V && er);
+        const int ekey = edge ? op.mode * 64 + q : -1000;
+        auto key = std::make_tuple(row[idx].lo, lo, ekey);
+        auto it = swsh_memo.find(key);
+        if (it != swsh_memo.end()) return it->second;
+        SwReg t = row[idx];
+        t.lo = var();
+        t.hi = var();
+        const char *fn = lo < 0 ? "__shfl_up_sync" : "__shfl_down_sync";
+        o << ind << "const unsigned " << t.lo << " = " << fn << "(KF_FULL, " << row[idx].lo << ", " << std::abs(lo) << ");\n";
+        o << ind << "const unsigned " << t.hi << " = " << fn << "(KF_FULL, " << row[idx].hi << ", " << std::abs(lo) << ");\n";
+        if (edge) {
+            std::string slo, shi;
+            int m;
+            if (q < 0) m = edge_map(op.mode, q);
+            else m = edge_map(op.mode, -(q - V) - 1);
+            if (m < 0) {
+                slo = shi = SwEmitter::lit(csub + row[0].B);
+            } else {
+                const SwReg &sr = q < 0 ? row[m] : row[V - 1 - m];
+                slo = sr.lo;
+                shi = sr.hi;
+            }
+            const std::string cond = q < 0 ? "x == 0" : "x == W - 4";
+            SwReg t2 = t;
+            t2.lo = var();
+            t2.hi = var();
+            o << ind << "const unsigned " << t2.lo << " = (" << cond << ") ? " << slo << " : " << t.lo << ";\n";
+            o << ind << "const unsigned " << t2.hi << " = (" << cond << ") ? " << shi << " : " << t.hi << ";\n";
+            t = t2;
+        }
+        swsh_memo[key] = t;
+        return t;
+    }
+    void kernel_sw(int k, int j, int u, const std::string &ind)
+    {
+        const Op &op = p->ops[k];
+        const int img = p->n_inputs + k;
+        SwEmitter e = swe(ind);
+        std::vector<SwLin> res(V);
+        if (op.kind == POINT) {
+            for (int v = 0; v < V; v++) {
+                std::vector<SwLin> loads;
+                for (int in : op.inputs) loads.push_back(SwEmitter::of(svalue(in, sl(in, HY(img) - HY(in), j), v, ind)));
+                res[v] = e.prog(op, loads);
+            }
+        } else {
+            const int in = op.inputs[0];
+            const int rx = op.mw / 2, ry = op.mh / 2;
+            auto mrow = [&](int dyp) { return ry + dir * dyp; };
+            const long long c = (long long)op.constant;
+            const Separable &sp = si.sep.at(k);
+            std::vector<SwLin> acc(V);
+            if (sp.ok) {
+                std::vector<SwLin> vl(V);
+                long long csum = 0;
+                for (double cc : sp.col) csum += (long long)cc;
+                for (int dy = -ry; dy <= ry; dy++) {   // mask-row order in both directions
+                    const int dyp = dir * dy;
+                    const long long cf = (long long)sp.col[mrow(dyp)];
+                    if (cf == 0) continue;
+                    bool isc = false;
+                    const int s = tap_slot(img, op, in, dyp, j, u, isc);
+                    for (int v = 0; v < V; v++)
+                        vl[v] = isc ? SwEmitter::add(vl[v], SwEmitter::cst(cf * c))
+                                    : SwEmitter::add(vl[v], SwEmitter::scale(SwEmitter::of(svalue(in, s, v, ind)), cf));
+                }
+                std::vector<SwReg> vs(V);
+                for (int v = 0; v < V; v++) vs[v] = e.mat(vl[v]);
+                for (int v = 0; v < V; v++)
+                    for (int dx = -rx; dx <= rx; dx++) {
+                        const long long rf = (long long)sp.row[dx + rx];
+                        if (rf == 0) continue;
+                        acc[v] = SwEmitter::add(acc[v], SwEmitter::scale(SwEmitter::of(at_col_sw(vs, v + dx, op, c * csum, ind)), rf));
+                    }
+            } else {
+                for (int dy = -ry; dy <= ry; dy++) {
+                    const int dyp = dir * dy;
+                    const int mr = mrow(dyp);
+                    bool any = false;
+                    for (int dx = -rx; dx <= rx; dx++) any |= op.mask[(size_t)mr * op.mw + dx + rx] != 0.0;
+                    if (!any) continue;
+                    bool isc = false;
+                    const int s = tap_slot(img, op, in, dyp, j, u, isc);
+                    std::vector<SwReg> row(V);
+                    if (!isc)
+                        for (int v = 0; v < V; v++) row[v] = svalue(in, s, v, ind);
+                    for (int dx = -rx; dx <= rx; dx++) {
+                        const long long m = (long long)op.mask[(size_t)mr * op.mw + dx + rx];
+                        if (m == 0) continue;
+                        for (int v = 0; v < V; v++)
+                            acc[v] = isc ? SwEmitter::add(acc[v], SwEmitter::cst(m * c))
+                                         : SwEmitter::add(acc[v], SwEmitter::scale(SwEmitter::of(at_col_sw(row, v + dx, op, c, ind)), m));
+                    }
+                }
+            }
+            for (int v = 0; v < V; v++) res[v] = op.prog.empty() ? acc[v] : e.prog(op, {acc[v]});
+        }
+        const int ws = sl(img, 0, j);
+        for (int v = 0; v < V; v++) {
+            SwReg r = e.sat_norm(res[v]);   // narrowing at the kernel boundary (R-16)
+            o << ind << ring(img, ws, v) << " = " << e.pack(r) << ";\n";
+            sw_memo[std::make_tuple(img, ws, v)] = r;
+        }
+    }
+
     // kernel k at iteration slot j: emits code, stores its V values into its
     // ring slot j, and memoises the unpacked values.
     void kernel(int k, int j, int u, const std::string &ind)
     {
+        if (si.swk.count(k)) {
+            kernel_sw(k, j, u, ind);
+            return;
+        }
         const Op &op = p->ops[k];
         const int img = p->n_inputs + k;
         std::vector<std::string> res(V);
@@ -854,6 +1271,8 @@ struct StreamGen {
         const int P = si.P, D = si.D, L = si.L;
         val_memo.clear();
         shfl_memo.clear();
+        sw_memo.clear();
+        swsh_memo.clear();
         o << ind.substr(2) << "{   // iteration " << uexpr << " + " << j << "\n";
         if (si.sring) {
             const int DS = si.DS;
@@ -896,7 +1315,8 @@ struct StreamGen {
         } else if (!si.vec) {
             for (int v = 0; v < V; v++) {
                 std::string val = f32 ? (pm ? value(simg, ss, v, ind) : ring(simg, ss, v))
-                                      : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
+                                      : si.swk.count(b.sink) ? ring(simg, ss, v)
+                                                             : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
                 o << ind << "    if (x + " << v << " < a.fx1) (" << orow << ")[" << v << "] = " << val << ";\n";
             }
         } else if (f32) {
@@ -905,7 +1325,8 @@ struct StreamGen {
             o << ");\n";
         } else {
             o << ind << "    kf_st4u(" << orow;
-            for (int v = 0; v < V; v++) o << ", kf_pack(" << val_memo[std::make_tuple(simg, ss, v)] << ")";
+            for (int v = 0; v < V; v++)
+                o << ", " << (si.swk.count(b.sink) ? ring(simg, ss, v) : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")");
             o << ");\n";
         }
         o << ind << "}\n";
@@ -1165,6 +1586,9 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
             si.depth[in] = std::max(si.depth[in], d);
         }
         if (op.kind == LOCAL) si.sep[k] = factor(op, p->dtype != KF_F32);
+        if (p->dtype == KF_U8X4 && env_int("KFUSE_SWAR", 1, 0, 1) &&
+            swar_feasible(op, op.kind == LOCAL ? si.sep[k] : Separable{}))
+            si.swk.insert(k);
     }
     for (auto &kv : si.depth) {
         bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
@@ -1195,10 +1619,10 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     }
     si.live_regs = live;
     // code size: scalar operations of one iteration (one body copy)
-    const int ch = p->dtype == KF_F32 ? 1 : 4;
     long long ops = 0;
     for (int k : b.kernels) {
         const Op &op = p->ops[k];
+        const int ch = p->dtype == KF_F32 ? 1 : si.swk.count(k) ? 2 : 4;   // SWAR: two channels per op
         if (op.kind == LOCAL) {
             int nnz = 0;
             for (double m : op.mask) nnz += m != 0.0;

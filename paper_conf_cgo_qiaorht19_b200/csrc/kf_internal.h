@@ -152,6 +152,7 @@ struct StreamInfo {
     std::map<int, int> hy;        // image -> rows needed around the sink row
     std::map<int, int> depth;     // image -> history depth (iterations)
     std::map<int, Separable> sep; // local kernel -> factorisation
+    std::set<int> swk;            // u8x4 kernels in SWAR form (two channels per 32-bit op)
 };
 
 std::string kernel_name(const BlockInfo &b, int block);

@@ -71,6 +71,57 @@ def exchange_halos(buf: torch.Tensor, band: Band, group=None) -> None:
         req.wait()
 
 
+def split_rows(band: Band) -> tuple[tuple[int, int], list[tuple[int, int]]]:
+    """Output rows of a band that need no halo row -- the core [row0 + t, row1 - b)
+    with t (b) = R when a neighbour exists above (below), else 0 -- and the edge
+    strips that do.  The core can run while the halo rows are in flight."""
+    t = band.halo if band.rank > 0 else 0
+    b = band.halo if band.rank < band.world - 1 else 0
+    c0, c1 = band.row0 + t, band.row1 - b
+    if c0 >= c1:
+        return (band.row0, band.row0), [(band.row0, band.row1)]
+    edges = [(r0, r1) for r0, r1 in ((band.row0, c0), (c1, band.row1)) if r1 > r0]
+    return (c0, c1), edges
+
+
+def run_step_overlapped(plan, band: Band, inputs, outputs, side_stream, group=None) -> None:
+    """One multi-GPU step with the exchange hidden behind the band's core rows
+    (SURVEY §8(e) "overlap"): the halo send/recv is posted first (NCCL runs on its
+    own stream), the core rows run on `side_stream` meanwhile, then the current
+    stream waits for the halo rows and computes the edge strips.  Output is
+    bit-identical to exchange_halos + run_band (border modes act at the global
+    edges in every call)."""
+    cur = torch.cuda.current_stream()
+    (c0, c1), edges = split_rows(band)
+    side_stream.wait_stream(cur)                      # inputs of this step are ready
+    reqs = []
+    if band.world > 1 and band.halo > 0:
+        reqs = _post_halos(inputs, band, group)
+    if c1 > c0:
+        with torch.cuda.stream(side_stream):
+            outs = [o[c0 - band.row0:c1 - band.row0] for o in outputs]
+            plan.run_band(c0, c1, inputs, band.in0, band.in1, outs, side_stream)
+    for r in reqs:
+        r.wait()
+    for r0, r1 in edges:
+        outs = [o[r0 - band.row0:r1 - band.row0] for o in outputs]
+        plan.run_band(r0, r1, inputs, band.in0, band.in1, outs, cur)
+    cur.wait_stream(side_stream)
+
+
+def _post_halos(inputs, band: Band, group=None) -> list:
+    ops = []
+    t, b, n = band.top, band.bottom, band.rows
+    for buf in inputs:
+        if band.rank > 0:
+            ops.append(dist.P2POp(dist.isend, buf[t:t + band.halo], band.rank - 1, group))
+            ops.append(dist.P2POp(dist.irecv, buf[0:t], band.rank - 1, group))
+        if band.rank < band.world - 1:
+            ops.append(dist.P2POp(dist.isend, buf[t + n - band.halo:t + n], band.rank + 1, group))
+            ops.append(dist.P2POp(dist.irecv, buf[t + n:t + n + b], band.rank + 1, group))
+    return dist.batch_isend_irecv(ops) if ops else []
+
+
 def run_band(plan, band: Band, inputs, outputs, stream=None) -> None:
     """inputs: device tensors holding rows [in0, in1) (halo exchanged);
     outputs: device tensors of band.rows rows."""

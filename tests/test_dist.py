@@ -48,7 +48,7 @@ def test_partition_rejects_band_thinner_than_halo():
         KD.partition(8, 4, 1, 3)
 
 
-def _worker(rank, world, port, H, W, halo, q):
+def _worker(rank, world, port, H, W, halo, q, posted=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -57,20 +57,25 @@ def _worker(rank, world, port, H, W, halo, q):
         buf = torch.full((band.in1 - band.in0, W), float("nan"))
         own = torch.from_numpy(full[band.row0:band.row1])
         buf[band.top:band.top + band.rows] = own
-        KD.exchange_halos(buf, band)
+        if posted:   # the overlapped step's non-blocking post (dist.run_step_overlapped)
+            for r in KD._post_halos([buf], band):
+                r.wait()
+        else:
+            KD.exchange_halos(buf, band)
         ok = bool(np.array_equal(buf.numpy(), full[band.in0:band.in1]))
         q.put((rank, ok))
     finally:
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("posted", [False, True])
 @pytest.mark.parametrize("world,H,halo", [(2, 37, 2), (3, 50, 6), (2, 9, 4)])
-def test_exchange_halos_gloo(world, H, halo):
+def test_exchange_halos_gloo(world, H, halo, posted):
     """After one exchange every rank holds exactly rows [in0, in1) of the global image."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, H, 23, halo, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, H, 23, halo, q, posted)) for r in range(world)]
     for p in procs:
         p.start()
     res = dict(q.get(timeout=120) for _ in procs)
@@ -78,3 +83,21 @@ def test_exchange_halos_gloo(world, H, halo):
         p.join(timeout=60)
         assert p.exitcode == 0
     assert all(res[r] for r in range(world)), res
+
+
+@pytest.mark.parametrize("H,world,halo", [(97, 3, 2), (100, 4, 6), (9, 2, 4), (50, 1, 3), (12, 3, 2)])
+def test_split_rows_core_and_edges(H, world, halo):
+    """The core rows need no halo row ([row0+R, row1-R) reads only owned rows) and
+    core + edge strips cover the band exactly once."""
+    for rank in range(world):
+        try:
+            b = KD.partition(H, world, rank, halo)
+        except ValueError:
+            continue
+        (c0, c1), edges = KD.split_rows(b)
+        rows = list(range(c0, c1)) + [y for r0, r1 in edges for y in range(r0, r1)]
+        assert sorted(rows) == list(range(b.row0, b.row1))
+        if c1 > c0:
+            lo = c0 - halo if rank > 0 else max(0, c0 - halo)
+            hi = c1 + halo if rank < world - 1 else min(H, c1 + halo)
+            assert (rank == 0 or lo >= b.row0) and (rank == world - 1 or hi <= b.row1)

@@ -225,6 +225,26 @@ def test_bands_bit_identical(wl, kind):
         np.testing.assert_array_equal(out.cpu().numpy(), full[r0:r1])
 
 
+@pytest.mark.parametrize("wl", ["harris", "deep10"])
+@pytest.mark.parametrize("rank,world", [(0, 3), (1, 3), (2, 3), (0, 1)])
+def test_overlapped_step_equals_full_run(wl, rank, world, monkeypatch):
+    """dist.run_step_overlapped (core rows on a side stream while the halo is in
+    flight, then the edge strips) reproduces the full run; the halo rows are
+    pre-filled here, so the NCCL post is stubbed out."""
+    from paper_conf_cgo_qiaorht19_b200 import dist as KD
+    spec = P.WORKLOADS[wl](200, 150)
+    ins = _inputs(spec, 12)
+    plan = make_plan(spec, "b200")
+    full = run_gpu(spec, plan, ins)[0]
+    band = KD.partition(spec["height"], world, rank, plan.halo_rows)
+    monkeypatch.setattr(KD, "_post_halos", lambda inputs, band, group=None: [])
+    d_in = [torch.from_numpy(np.ascontiguousarray(a[band.in0:band.in1])).cuda() for a in ins]
+    out = torch.empty((band.rows,) + full.shape[1:], dtype=d_in[0].dtype, device="cuda")
+    KD.run_step_overlapped(plan, band, d_in, [out], torch.cuda.Stream())
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(out.cpu().numpy(), full[band.row0:band.row1])
+
+
 def test_launch_count_matches_blocks():
     spec = P.harris(512, 512)
     for kind, n in (("unfused", 9), ("paper", 6), ("b200", 1)):
