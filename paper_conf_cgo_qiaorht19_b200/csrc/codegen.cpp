@@ -234,6 +234,7 @@ struct SwEmitter {
     std::ostringstream *o = nullptr;   // null: interval-only dry run (feasibility)
     int *tmp = nullptr;
     std::string ind;
+    std::string lut_sym;               // device table of the kernel being emitted (LUT ops)
     std::string var() { return "w" + std::to_string((*tmp)++); }
     static std::string lit(long long v)   // v * 0x10001 as an unsigned literal (mod 2^32)
     {
@@ -372,6 +373,35 @@ struct SwEmitter {
     }
     // kernel boundary: saturate to [0, 255] and normalise to bias 0 (R-16)
     SwReg sat_norm(const SwLin &l) { return mat(of(clamp(mat(l), 0, 255))); }
+    // table gather per channel (index clamped to the table, as kf_lut does);
+    // entries must fit a lane: [0, 65535]
+    SwReg lut(const SwReg &x0, const std::vector<int> &tab)
+    {
+        if (tab.empty()) throw SwFail{};
+        const long long n = (long long)tab.size();
+        const long long tmin = *std::min_element(tab.begin(), tab.end());
+        const long long tmax = *std::max_element(tab.begin(), tab.end());
+        if (tmin < 0 || tmax > 65535 || n > 65536) throw SwFail{};
+        SwReg x = mat(of(clamp(x0, 0, n - 1)));   // bias 0 lanes = indices
+        SwReg r;
+        r.B = 0;
+        r.vlo = tmin;
+        r.vhi = tmax;
+        if (o) {
+            std::string t[4];
+            for (int c = 0; c < 4; c++) {
+                t[c] = var();
+                const std::string &w = c < 2 ? x.lo : x.hi;
+                *o << ind << "const unsigned " << t[c] << " = (unsigned)__ldg(" << lut_sym << " + "
+                   << (c % 2 ? "(" + w + " >> 16)" : "(" + w + " & 0xffffu)") << ");\n";
+            }
+            r.lo = var();
+            r.hi = var();
+            *o << ind << "const unsigned " << r.lo << " = __byte_perm(" << t[0] << ", " << t[1] << ", 0x5410);\n";
+            *o << ind << "const unsigned " << r.hi << " = __byte_perm(" << t[2] << ", " << t[3] << ", 0x5410);\n";
+        }
+        return r;
+    }
     SwReg unpack(const std::string &u)
     {
         SwReg r;
@@ -439,7 +469,8 @@ struct SwEmitter {
                 break;
             }
             case KF_OP_SAT_U8: st.push_back(of(clamp(mat(pop()), 0, 255))); break;
-            default: throw SwFail{};   // DIV, ABS, SELECT_GT, LUT, POW, ...
+            case KF_OP_LUT: st.push_back(of(lut(mat(pop()), op.lut))); break;
+            default: throw SwFail{};   // DIV, ABS, SELECT_GT, POW, ...
             }
         }
         return st.back();
@@ -929,6 +960,7 @@ struct StreamGen {
 
     // ---- SWAR form of u8x4 kernels
     SwEmitter swe(const std::string &ind) { SwEmitter e; e.o = &o; e.tmp = &tmp; e.ind = ind; return e; }
+    std::string lut_sym(int k) const { return "kf_lut_" + std::to_string(block) + "_" + std::to_string(k); }
     // value of image img at ring slot s, column v (bias 0, [0, 255]): memo or unpack
     SwReg svalue(int img, int s, int v, const std::string &ind)
     {
@@ -986,6 +1018,7 @@ struct StreamGen {
         const Op &op = p->ops[k];
         const int img = p->n_inputs + k;
         SwEmitter e = swe(ind);
+        e.lut_sym = lut_sym(k);
         std::vector<SwLin> res(V);
         if (op.kind == POINT) {
             for (int v = 0; v < V; v++) {
