@@ -170,7 +170,7 @@ def run_reference(args, cfg_name, spec) -> None:
         "impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot / args.steps * 1e3, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-        "data": DATA, "config": config_dict(cfg_name, spec, "unfused-oracle"),
+        "data": DATA, "config": config_dict(cfg_name, spec, "unfused-oracle", {"l2": "n/a: host oracle"}),
         "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
         "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }))

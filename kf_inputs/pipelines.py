@@ -208,6 +208,32 @@ def blur(width: int, height: int, mode: str = "clamp") -> dict:
     return p.spec()
 
 
+def swar_stress(W, H, mode="mirror"):
+    """u8x4 kernels on both sides of the SWAR interval check: linear forms with
+    negative ranges, MIN/MAX of differently biased values, NEG/SHL, clamps, a short
+    LUT with entries above 255, a CONSTANT border at 255 -- and kernels that must
+    fall back to int32 (a 16-bit-overflowing mask, ABS, DIV, SELECT, a variable
+    product)."""
+    ACC = L(0)
+    p = Pipeline("swar_stress", W, H, "u8x4")
+    i = p.input()
+    a = p.local("a", i, [[1, -2, 1], [-2, 4, -2], [1, -2, 1]], "constant", constant=255.0,
+                post=[ACC, C(64), ADD, SHR(2), SAT])
+    b = p.point("b", [i, a], [L(0), L(1), SUB, NEG, L(0), MAX, C(1), op("SHL", 2), ADD, SHR(3), SAT])
+    c = p.point("c", [a, b], [L(0), C(3), MUL, L(1), MIN, C(10), C(200), CLAMP])
+    d = p.point("d", [c], [L(0), LUT], lut=[(7 * v) % 301 for v in range(100)])
+    big = [[60] * 5 for _ in range(5)]
+    e = p.local("e", d, big, mode, post=[ACC, SHR(12), SAT])                 # 16-bit overflow: int32
+    f = p.point("f", [e, b], [L(0), L(1), SUB, ABS, C(255), MIN])           # ABS: int32
+    g = p.point("g", [f, c], [L(0), C(7), MUL, L(1), C(1), ADD, DIV, SAT])  # DIV: int32
+    h = p.point("h", [g, a, b, d], [L(0), L(1), L(2), L(3), SELGT])          # SELECT: int32
+    k = p.point("k", [h, g], [L(0), L(1), MUL, SHR(8), SAT])                 # variable product: int32
+    m = p.local("m", k, [[1, 2, 1], [2, 4, 2], [1, 2, 1]], "constant", constant=255.0,
+                post=[ACC, C(8), ADD, SHR(4), SAT])
+    p.output(m)
+    return p.spec()
+
+
 def fig4(mode: str = "clamp") -> dict:
     """Fig. 4: two unnormalised 3x3 Gaussian local kernels on a 5x5 image."""
     p = Pipeline("fig4", 5, 5, "f32")

@@ -214,3 +214,27 @@ def test_exact_planner_size_limit():
     p.output(x)
     with pytest.raises(K.KfError):
         K.Pipeline.from_spec(p.spec()).plan_exact("paper")
+
+
+def test_swar_form_chosen_by_interval_analysis():
+    """u8x4 codegen: kernels whose lanes provably fit 16 bits run
+    two channels per op (PRMT-unpacked SWAR); a 16-bit-overflowing mask, ABS, DIV,
+    SELECT and a variable product fall back to per-channel int32; KFUSE_SWAR=0
+    turns the form off."""
+    spec = P.swar_stress(64, 48)
+    plan = K.Pipeline.from_spec(spec).plan_unfused()
+    form = {}
+    for b in range(plan.num_launches):
+        body = plan.source(b).split("_fast_di(")[1]
+        form[spec["ops"][b]["name"]] = "swar" if "__byte_perm" in body else "int32"
+    assert form == {"a": "swar", "b": "swar", "c": "swar", "d": "swar", "e": "int32", "f": "int32",
+                    "g": "int32", "h": "int32", "k": "int32", "m": "swar"}
+    os.environ["KFUSE_SWAR"] = "0"
+    try:
+        plan = K.Pipeline.from_spec(spec).plan_unfused()
+        assert all("__byte_perm" not in plan.source(b).split("_fast_di(")[1] for b in range(plan.num_launches))
+    finally:
+        del os.environ["KFUSE_SWAR"]
+    c4, _ = P.config("C4")
+    src = K.Pipeline.from_spec(c4).plan_fusion("b200").source(0).split("_fast_di(")[1]
+    assert "kf_unpack" not in src and "kf_lut(" not in src   # all ten deep10 kernels in SWAR form

@@ -249,3 +249,23 @@ def test_launch_count_matches_blocks():
     spec = P.harris(512, 512)
     for kind, n in (("unfused", 9), ("paper", 6), ("b200", 1)):
         assert make_plan(spec, kind).num_launches == n
+
+
+# ------------------------------------------------ u8x4 SWAR form
+
+
+@pytest.mark.parametrize("kind", ["unfused", "paper", "b200"])
+@pytest.mark.parametrize("size", [(67, 41), (256, 96)])
+def test_swar_matches_int32_and_oracle(kind, size, monkeypatch):
+    """The SWAR form and the per-channel int32 form give the same bytes, and both
+    equal the oracle (u8x4 parity is bit-exact)."""
+    spec = P.swar_stress(*size)
+    ins = _inputs(spec, 21)
+    ref = O.run(spec, ins)[spec["outputs"][0]]
+    outs = {}
+    for sw in ("1", "0"):
+        monkeypatch.setenv("KFUSE_SWAR", sw)
+        plan = make_plan(spec, kind)
+        outs[sw] = run_gpu(spec, plan, ins)[0]
+        check(spec, outs[sw], ref, f"swar={sw} {kind} {size}")
+    np.testing.assert_array_equal(outs["1"], outs["0"])
