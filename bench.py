@@ -398,6 +398,31 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms = float(ms.item())
     px = W * Htot
+    # end to end through the public API: each step uploads the band's own rows
+    # from pinned host memory, runs the overlapped step (halo exchange + fused
+    # kernels) and downloads the band's output; max over ranks of the wall time
+    hin = torch.from_numpy(host).pin_memory()
+    hout = torch.empty(oshape, dtype=tdt).pin_memory()
+    t, n = band.top, band.rows
+    e2e_steps = max(3, min(args.steps, 20))
+
+    def e2e_step():
+        ins[0][t:t + n].copy_(hin[t:t + n], non_blocking=True)
+        KD.run_step_overlapped(plan, band, [ins[0]], [outs[0]], side)
+        hout.copy_(outs[0], non_blocking=True)
+        torch.cuda.current_stream().synchronize()
+
+    e2e_step()
+    dist.barrier()
+    tw = time.perf_counter()
+    for _ in range(e2e_steps):
+        e2e_step()
+    e2e_s = torch.tensor([(time.perf_counter() - tw) / e2e_steps], device="cuda")
+    dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX)
+    e2e = {"value": round(px / float(e2e_s.item()) / 1e6, 1), "unit": UNIT,
+           "h2d_bytes_per_step": int(n * hin[0].numel() * hin.element_size()),
+           "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps,
+           "note": "per rank, max over ranks"}
     if rank == 0:
         ab = ALG_BYTES.get(gspec["name"], {}).get(args.plan) or 8
         peaks = load_peaks()
@@ -413,7 +438,7 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
                          "frac": round(ach / peaks["hbm_gbs"], 4), "traffic": None,
                          "peak_source": peaks["source"], "note": "per GPU, step time incl. halo exchange"},
             "cpu_baseline": None,
-            "e2e": None,
+            "e2e": e2e,
             "gpu_launches": args.steps * plan.num_launches, "clocks": cs.summary(),
         }))
     dist.destroy_process_group()
@@ -429,6 +454,7 @@ def main():
     ap.add_argument("--plan", default="b200", choices=list(PLANS))
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-extra", action="store_true", help="skip the other BASELINE configs")
+    ap.add_argument("--force-multi", action="store_true", help="run the row-band (torchrun) path even at world 1")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     from kf_inputs import pipelines as P
@@ -437,7 +463,7 @@ def main():
         run_reference(args, args.config, spec)
         return
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    if world > 1:
+    if world > 1 or args.force_multi:
         bench_multi(args, args.config, spec, seed)
     else:
         bench_single(args, args.config, spec, seed)

@@ -772,6 +772,7 @@ struct StreamGen {
     std::string var() { return "v" + std::to_string(tmp++); }
     int HY(int img) const { return si.hy.at(img); }
     int NR() const { return pm ? V / 2 : V; }                         // ring registers per row
+    int NRi(int img) const { return si.swring.count(img) ? 2 * V : NR(); }   // SWAR rings: (lo, hi) per pixel
     std::string RDT() const { return pm ? "F2" : RT(); }               // ring register type
     static int md(int a, int m) { return ((a % m) + m) % m; }
     bool is_ext(int img) const { return std::binary_search(b.ext.begin(), b.ext.end(), img); }
@@ -809,7 +810,11 @@ struct StreamGen {
         std::string r = ring(img, s, v);
         if (!f32) {
             std::string t = var();
-            o << ind << "const I4 " << t << " = kf_unpack(" << r << ");\n";
+            if (si.swring.count(img))
+                o << ind << "const I4 " << t << " = kf_unpack_sw(" << ring(img, s, 2 * v) << ", " << ring(img, s, 2 * v + 1)
+                  << ");\n";
+            else
+                o << ind << "const I4 " << t << " = kf_unpack(" << r << ");\n";
             r = t;
         }
         val_memo[key] = r;
@@ -967,6 +972,13 @@ struct StreamGen {
         auto key = std::make_tuple(img, s, v);
         auto it = sw_memo.find(key);
         if (it != sw_memo.end()) return it->second;
+        if (si.swring.count(img)) {   // SWAR ring: already unpacked (bias 0, [0, 255])
+            SwReg r;
+            r.lo = ring(img, s, 2 * v);
+            r.hi = ring(img, s, 2 * v + 1);
+            sw_memo[key] = r;
+            return r;
+        }
         SwReg r = swe(ind).unpack(ring(img, s, v));
         sw_memo[key] = r;
         return r;
@@ -1081,7 +1093,12 @@ struct StreamGen {
         const int ws = sl(img, 0, j);
         for (int v = 0; v < V; v++) {
             SwReg r = e.sat_norm(res[v]);   // narrowing at the kernel boundary (R-16)
-            o << ind << ring(img, ws, v) << " = " << e.pack(r) << ";\n";
+            if (si.swring.count(img)) {
+                o << ind << ring(img, ws, 2 * v) << " = " << r.lo << ";\n";
+                o << ind << ring(img, ws, 2 * v + 1) << " = " << r.hi << ";\n";
+            } else {
+                o << ind << ring(img, ws, v) << " = " << e.pack(r) << ";\n";
+            }
             sw_memo[std::make_tuple(img, ws, v)] = r;
         }
     }
@@ -1247,6 +1264,11 @@ struct StreamGen {
             if (pm) {
                 o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
                 o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
+            } else if (si.swring.count(img)) {
+                for (int v = 0; v < V; v++) {
+                    o << ind << ring(img, rs, 2 * v) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4140);\n";
+                    o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4342);\n";
+                }
             } else {
                 for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
             }
@@ -1254,6 +1276,11 @@ struct StreamGen {
             for (int q = 0; q < V / 2; q++)
                 o << ind << ring(img, rs, q) << " = make_float2(__ldg(" << ptr << " + cl" << 2 * q << "), __ldg(" << ptr
                   << " + cl" << 2 * q + 1 << "));\n";
+        } else if (si.swring.count(img)) {
+            for (int v = 0; v < V; v++) {
+                o << ind << ring(img, rs, 2 * v) << " = __byte_perm(__ldg(" << ptr << " + cl" << v << "), 0u, 0x4140);\n";
+                o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(__ldg(" << ptr << " + cl" << v << "), 0u, 0x4342);\n";
+            }
         } else {
             for (int v = 0; v < V; v++)
                 o << ind << ring(img, rs, v) << " = __ldg(" << ptr << " + cl" << v << ");\n";
@@ -1292,6 +1319,12 @@ struct StreamGen {
         if (pm) {
             o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
             o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
+        } else if (si.swring.count(img)) {
+            const char *c[4] = {"x", "y", "z", "w"};
+            for (int v = 0; v < V; v++) {
+                o << ind << ring(img, rs, 2 * v) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4140);\n";
+                o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4342);\n";
+            }
         } else {
             const char *c[4] = {"x", "y", "z", "w"};
             for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
@@ -1369,7 +1402,7 @@ struct StreamGen {
             for (int k : b.kernels) imgs.insert(p->n_inputs + k);
             for (int img : imgs)
                 for (int a = ring_len(img) - 1; a >= 1; a--)
-                    for (int v = 0; v < NR(); v++) o << ind << ring(img, a, v) << " = " << ring(img, a - 1, v) << ";\n";
+                    for (int v = 0; v < NRi(img); v++) o << ind << ring(img, a, v) << " = " << ring(img, a - 1, v) << ";\n";
         }
         o << ind.substr(2) << "}\n";
     }
@@ -1420,7 +1453,7 @@ struct StreamGen {
             o << "    " << RDT();
             bool first = true;
             for (int s = 0; s < ring_len(img); s++)
-                for (int v = 0; v < NR(); v++) {
+                for (int v = 0; v < NRi(img); v++) {
                     o << (first ? " " : ", ") << ring(img, s, v) << (pm ? " = kf2(0.0f)" : " = 0");
                     first = false;
                 }
@@ -1600,6 +1633,25 @@ int env_int(const char *name, int dflt, int lo, int hi)
     return std::min(hi, std::max(lo, v));
 }
 
+// Code-size weight of a program: SASS instructions its opcodes expand to
+// (accurate libdevice powf / logf / expf / sqrtf / division are inline
+// sequences of tens of instructions; fitted to cuobjdump counts on sm_100a).
+static int prog_size(const Op &op)
+{
+    int n = 0;
+    for (const Instr &in : op.prog) {
+        switch (in.op) {
+        case KF_OP_POW: n += 80; break;
+        case KF_OP_LOG: n += 30; break;
+        case KF_OP_EXP: n += 25; break;
+        case KF_OP_SQRT: n += 8; break;
+        case KF_OP_DIV: n += 15; break;
+        default: n += 1;
+        }
+    }
+    return n;
+}
+
 StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
 {
     StreamInfo si;
@@ -1650,6 +1702,34 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
         live += (kv.second + (ext && !si.sring ? si.D : 0)) * kStreamV;
     }
+    // SWAR rings: a u8x4 image read at several rows per
+    // iteration by SWAR local kernels keeps its ring unpacked -- (lo, hi) per
+    // pixel, written once -- instead of packed uchar4 re-unpacked (2 PRMT per
+    // pixel) at every row use.  Costs depth x V more registers; deepest first,
+    // under a cap on the live ring registers.
+    const int live_packed = live;
+    if (p->dtype == KF_U8X4 && env_int("KFUSE_SWRING", 1, 0, 1)) {
+        const int cap = env_int("KFUSE_SWRING_CAP", 164, 0, 1024);
+        std::vector<std::pair<int, int>> cand;   // (depth, image)
+        for (auto &kv : si.depth) {
+            const int img = kv.first;
+            if (img == p->n_inputs + b.sink || kv.second < 3) continue;
+            const bool ext = std::binary_search(b.ext.begin(), b.ext.end(), img);
+            if (!ext && !si.swk.count(img - p->n_inputs)) continue;   // producer must be SWAR (or a load)
+            bool vert = false;
+            for (int k : b.kernels)
+                if (si.swk.count(k) && p->ops[k].kind == LOCAL && p->ops[k].ry() >= 1 && p->ops[k].inputs[0] == img)
+                    vert = true;
+            if (vert) cand.push_back({kv.second, img});
+        }
+        std::sort(cand.begin(), cand.end(), [](auto &a, auto &b2) { return a.first != b2.first ? a.first > b2.first : a.second < b2.second; });
+        for (auto &c : cand) {
+            const int extra = c.first * kStreamV;
+            if (live + extra > cap) continue;
+            live += extra;
+            si.swring.insert(c.second);
+        }
+    }
     si.live_regs = live;
     // code size: scalar operations of one iteration (one body copy)
     long long ops = 0;
@@ -1663,9 +1743,9 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
             int taps = sp.ok ? (int)(std::count_if(sp.col.begin(), sp.col.end(), [](double c) { return c != 0.0; }) +
                                      std::count_if(sp.row.begin(), sp.row.end(), [](double c) { return c != 0.0; }))
                              : nnz;
-            ops += (long long)(taps + 2 * op.rx() + (int)op.prog.size()) * kStreamV * ch;
+            ops += (long long)(taps + 2 * op.rx() + prog_size(op)) * kStreamV * ch;
         } else {
-            ops += (long long)op.prog.size() * kStreamV * ch;
+            ops += (long long)prog_size(op) * kStreamV * ch;
         }
     }
     si.iter_ops = ops;
@@ -1688,7 +1768,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     if (si.rolled) si.edge_v = false;
     si.edge_l = !rep && hfit && p->W >= 4 * kStreamV;
     si.edge_r = si.edge_l && si.vec;
-    si.ok = b.Rx <= 2 * kStreamV * 4 && live <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
+    si.ok = b.Rx <= 2 * kStreamV * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
     return si;
 }
 

@@ -72,6 +72,11 @@ __device__ __forceinline__ I4 kf_unpack(unsigned u)
 {
     return I4{(int)(u & 0xffu), (int)((u >> 8) & 0xffu), (int)((u >> 16) & 0xffu), (int)(u >> 24)};
 }
+// a pixel in SWAR form (two channels per 16-bit lane pair, bias 0) -> I4
+__device__ __forceinline__ I4 kf_unpack_sw(unsigned lo, unsigned hi)
+{
+    return I4{(int)(lo & 0xffffu), (int)(lo >> 16), (int)(hi & 0xffffu), (int)(hi >> 16)};
+}
 __device__ __forceinline__ int kf_sat(int v) { return min(max(v, 0), 255); }
 __device__ __forceinline__ unsigned kf_pack(I4 a)
 {

@@ -153,6 +153,7 @@ struct StreamInfo {
     std::map<int, int> depth;     // image -> history depth (iterations)
     std::map<int, Separable> sep; // local kernel -> factorisation
     std::set<int> swk;            // u8x4 kernels in SWAR form (two channels per 32-bit op)
+    std::set<int> swring;         // u8x4 images whose ring holds the unpacked SWAR (lo, hi) pair
 };
 
 std::string kernel_name(const BlockInfo &b, int block);
