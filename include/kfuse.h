@@ -227,7 +227,7 @@ kf_status kf_run(kf_pipeline *p, const kf_plan *plan, const void *const *d_input
 
 /* End-to-end call with HOST buffers: copies inputs host->device, runs, copies
  * outputs device->host, synchronises `stream`.  The image is processed in up to
- * 16 row bands on three engines: the H2D copy of band k+1's input rows, the
+ * 8 row bands on three engines: the H2D copy of band k+1's input rows, the
  * kernels of band k (kf_run_band semantics: border modes act at the global
  * edges, so the result equals kf_run's bit for bit) and the D2H copy of band
  * k-1's output rows overlap.  REPEAT plans run as one band.  Host buffers

@@ -165,7 +165,7 @@ struct CompiledBlock {
     }
 };
 
-constexpr int kHostBands = 16;  // kf_run_host pipeline depth (row bands)
+constexpr int kHostBands = 8;   // kf_run_host pipeline depth (row bands; 16 measured slower)
 
 struct Runtime {
     std::map<uint64_t, std::shared_ptr<CompiledBlock>> modules;   // by source hash

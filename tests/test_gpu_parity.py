@@ -269,3 +269,32 @@ def test_swar_matches_int32_and_oracle(kind, size, monkeypatch):
         outs[sw] = run_gpu(spec, plan, ins)[0]
         check(spec, outs[sw], ref, f"swar={sw} {kind} {size}")
     np.testing.assert_array_equal(outs["1"], outs["0"])
+
+
+def test_c5_full_size_and_four_bands():
+    """C5 (Harris 16384^2 f32, the multi-GPU config) at full size on one GPU:
+    sampled outputs against the recursive oracle, and the 4-band decomposition
+    (the 4-GPU row bands of §8(e), each band from its own input rows + halo)
+    bit-identical to the whole-image run."""
+    from paper_conf_cgo_qiaorht19_b200 import dist as KD
+    spec, seed = P.config("C5")
+    W, H = spec["width"], spec["height"]
+    img = _inputs(spec, seed)[0]
+    plan = make_plan(spec, "b200")
+    d_in = torch.from_numpy(img).cuda()
+    full = torch.empty((H, W), dtype=torch.float32, device="cuda")
+    plan.run([d_in], [full])
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(5)
+    ys, xs = _sample_points(W, H, rng, n=800)
+    ref = O.eval_points(spec, [img], spec["outputs"][0], ys, xs)
+    got = full[torch.from_numpy(ys).cuda(), torch.from_numpy(xs).cuda()].cpu().numpy().astype(np.float64)
+    assert np.abs(got - ref).max() / np.abs(ref).max() <= TOL
+    for r in range(4):
+        band = KD.partition(H, 4, r, plan.halo_rows)
+        b_in = d_in[band.in0:band.in1].clone()
+        b_out = torch.empty((band.rows, W), dtype=torch.float32, device="cuda")
+        KD.run_band(plan, band, [b_in], [b_out])
+        torch.cuda.synchronize()
+        assert torch.equal(b_out, full[band.row0:band.row1]), f"band {r} differs"
+        del b_in, b_out
