@@ -358,9 +358,10 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     from paper_conf_cgo_qiaorht19_b200 import dist as KD
     from paper_conf_cgo_qiaorht19_b200 import kfuse as K
 
-    dist.init_process_group("nccl")
+    # KFUSE_DIST_BACKEND=gloo and KFUSE_BENCH_DEVICE=0 let a 2-rank smoke run share one GPU (tests only)
+    dist.init_process_group(os.environ.get("KFUSE_DIST_BACKEND", "nccl"))
     rank, world = dist.get_rank(), dist.get_world_size()
-    dev = int(os.environ.get("LOCAL_RANK", rank))
+    dev = int(os.environ.get("KFUSE_BENCH_DEVICE", os.environ.get("LOCAL_RANK", rank)))
     torch.cuda.set_device(dev)
     W, Hb = spec["width"], spec["height"]
     Htot = Hb * world                                 # weak scaling: one band per GPU
@@ -375,42 +376,77 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     ins = [torch.from_numpy(host).cuda() for _ in range(nsets)]
     oshape = (band.rows, W) if gspec["dtype"] == "f32" else (band.rows, W, 4)
     outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(nsets)]
-    stream = torch.cuda.current_stream()
-
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
     side = torch.cuda.Stream()
+    # halo transport: peer memory (CUDA IPC mappings over NVLink, device-counter
+    # sync, whole steps captured in a CUDA graph) or NCCL send/recv (eager)
+    mode = os.environ.get("KFUSE_HALO", "peer")
+    halo, note = None, ""
+    if mode == "peer":
+        try:
+            halo = KD.PeerHalo(band, ins)
+        except Exception as e:   # e.g. no IPC between the ranks: fall back to NCCL
+            mode, note = "nccl", f"peer setup failed ({type(e).__name__}: {e}); "
+    (c0, c1), edges = KD.split_rows(band)
+    exch = halo is not None and (halo.up is not None or halo.down is not None)
+    launches_per_step = plan.num_launches * ((1 if c1 > c0 else 0) + len(edges)) + (2 if exch else 0)
 
-    def step(i):   # halo exchange (NCCL) overlapped with the band's core rows
-        KD.run_step_overlapped(plan, band, [ins[i % nsets]], [outs[i % nsets]], side)
+    def step(i):
+        if mode == "peer":   # core rows || (signal, halo pull over peer loads), then the edge strips
+            halo.step(plan, i % nsets, [outs[i % nsets]], stream, side)
+        else:                # NCCL send/recv overlapped with the core rows
+            KD.run_step_overlapped(plan, band, [ins[i % nsets]], [outs[i % nsets]], side)
 
     for i in range(args.warmup):
         step(i)
     torch.cuda.synchronize()
+    graph = None
+    if mode == "peer":   # every rank captures the same steps; the counters synchronise the replays
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=stream):
+            for i in range(args.steps):
+                step(i)
+        torch.cuda.synchronize()
     dist.barrier()
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(dev) as cs:
-        t0.record()
-        for i in range(args.steps):
-            step(i)
-        t1.record()
+        t0.record(stream)
+        if graph is not None:
+            graph.replay()
+        else:
+            for i in range(args.steps):
+                step(i)
+        t1.record(stream)
         torch.cuda.synchronize()
     dist.barrier()
     ms = torch.tensor([t0.elapsed_time(t1) / args.steps], device="cuda")
     dist.all_reduce(ms, op=dist.ReduceOp.MAX)
     ms = float(ms.item())
+    if halo is not None:
+        bad = torch.tensor([halo.errors()], device="cuda")
+        dist.all_reduce(bad, op=dist.ReduceOp.MAX)
+        if int(bad.item()):
+            raise RuntimeError("peer halo: a counter wait timed out")
     px = W * Htot
     # end to end through the public API: each step uploads the band's own rows
-    # from pinned host memory, runs the overlapped step (halo exchange + fused
-    # kernels) and downloads the band's output; max over ranks of the wall time
+    # from pinned host memory, runs the step (halo exchange + fused kernels) and
+    # downloads the band's output; max over ranks of the wall time
     hin = torch.from_numpy(host).pin_memory()
     hout = torch.empty(oshape, dtype=tdt).pin_memory()
     t, n = band.top, band.rows
     e2e_steps = max(3, min(args.steps, 20))
 
     def e2e_step():
+        if halo is not None:
+            halo.wait_consumed(stream)        # the neighbours pulled the previous rows
         ins[0][t:t + n].copy_(hin[t:t + n], non_blocking=True)
-        KD.run_step_overlapped(plan, band, [ins[0]], [outs[0]], side)
+        if halo is not None:
+            halo.step(plan, 0, [outs[0]], stream, side)
+        else:
+            KD.run_step_overlapped(plan, band, [ins[0]], [outs[0]], side)
         hout.copy_(outs[0], non_blocking=True)
-        torch.cuda.current_stream().synchronize()
+        stream.synchronize()
 
     e2e_step()
     dist.barrier()
@@ -423,6 +459,8 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
            "h2d_bytes_per_step": int(n * hin[0].numel() * hin.element_size()),
            "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps,
            "note": "per rank, max over ranks"}
+    how = ("peer-memory halo pull (CUDA IPC / NVLink P2P, device-counter sync), steps replayed from a CUDA graph"
+           if mode == "peer" else "NCCL send/recv overlapped with the core rows")
     if rank == 0:
         ab = ALG_BYTES.get(gspec["name"], {}).get(args.plan) or 8
         peaks = load_peaks()
@@ -432,15 +470,18 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": DATA,
             "config": config_dict(cfg_name, gspec, args.plan,
-                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows via NCCL send/recv overlapped with the core rows",
+                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows: {note}{how}",
                                    "band": f"{Hb}x{W} per GPU"}),
             "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
                          "frac": round(ach / peaks["hbm_gbs"], 4), "traffic": None,
                          "peak_source": peaks["source"], "note": "per GPU, step time incl. halo exchange"},
             "cpu_baseline": None,
             "e2e": e2e,
-            "gpu_launches": args.steps * plan.num_launches, "clocks": cs.summary(),
+            "gpu_launches": args.steps * launches_per_step, "clocks": cs.summary(),
         }))
+    if halo is not None:   # drop the peer mappings on every rank before any rank frees its buffers
+        halo.close()
+        dist.barrier()
     dist.destroy_process_group()
 
 

@@ -249,6 +249,35 @@ kf_status kf_run_band(kf_pipeline *p, const kf_plan *plan, int32_t row0, int32_t
                       const void *const *d_in_band, int32_t in_row0, int32_t in_row1,
                       void *const *d_out_band, void *stream);
 
+/* ---- multi-GPU halo rows over peer memory (NVLink P2P) ------------------
+ * The north star's "halo rows ... read from peer memory over NVLink"
+ * (BASELINE.json), as three stream-ordered, CUDA-graph-capturable
+ * kernels synchronised by monotonic uint32 counters in device memory (no host
+ * collective per step).  Pointers may be peer mappings (CUDA IPC) of another
+ * GPU's memory; the caller owns every buffer.  Counters compare wrap-safe.
+ * Every wait polls at most spin_limit times (~0.1 us each), then sets *err = 1
+ * and gives up (a missing neighbour is an error, not a hang).  Up to 4
+ * counters / segments per call; KF_ERR_ARG otherwise, KF_ERR_CUDA if the
+ * launch fails. */
+
+/* Release-increments each counter flags[i] (typically in the neighbours'
+ * memory: "my rows of this step are ready"), after everything queued before
+ * it on `stream`; increments *sent (local, nullable). */
+kf_status kf_peer_signal(uint32_t *const *flags, int32_t n, uint32_t *sent, void *stream);
+
+/* For each segment i: wait until *flag[i] passes *seen[i], copy bytes[i] bytes
+ * from src[i] (the neighbour's boundary rows) to dst[i] (the local halo rows),
+ * set *seen[i] += 1, then release-increment ack[i] (the neighbour's "consumed"
+ * counter; ack may be null). */
+kf_status kf_peer_pull(int32_t n, void *const *dst, const void *const *src, const int64_t *bytes,
+                       uint32_t *const *flag, uint32_t *const *seen, uint32_t *const *ack, uint32_t *err,
+                       int64_t spin_limit, void *stream);
+
+/* Wait until every *counter[i] reaches *target[i] (e.g. both neighbours acked
+ * every signal before the own rows are overwritten). */
+kf_status kf_peer_wait(int32_t n, uint32_t *const *counter, uint32_t *const *target, uint32_t *err,
+                       int64_t spin_limit, void *stream);
+
 /* Thread-local message of the last failing call on this thread. */
 const char *kf_last_error(void);
 /* Library version string. */

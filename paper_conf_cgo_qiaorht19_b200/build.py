@@ -21,7 +21,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-Wall",
          "-I", os.path.join(ROOT, "include"), "-I", CSRC]
-SOURCES = ["capi.cpp", "graph.cpp", "planner.cpp", "codegen.cpp", "runtime.cu"]
+SOURCES = ["capi.cpp", "graph.cpp", "planner.cpp", "codegen.cpp", "runtime.cu", "peer.cu"]
 
 
 def _embed_header() -> str:

@@ -197,6 +197,158 @@ struct ProgEmitter {
         };
         return ev(st.back());
     }
+
+    // Deferred power-of-two scaling: a packed value may be held
+    // as `stored` with true value = stored x 2^e, e a compile-time exponent.
+    // Scaling by a power of two is exact in binary floating point (away from
+    // overflow and subnormals), so (a 2^e)(b 2^f) = ab 2^(e+f) and
+    // a 2^e + b 2^e = (a + b) 2^e hold bit for bit: a normalised mask's 1/16
+    // is applied once at the end of the chain instead of at every stage.
+    struct Val {
+        std::string x;      // F2 expression (empty for a constant)
+        int e = 0;
+        bool isc = false;
+        double c = 0.0;
+    };
+    static std::string lit2(double c, int e) { return "kf2(" + fconst(std::ldexp((double)(float)c, -e)) + ")"; }
+    static bool pow2(double c, int &k)
+    {
+        if (c <= 0.0) return false;
+        int ex = 0;
+        const double m = std::frexp(c, &ex);
+        if (m != 0.5) return false;
+        k = ex - 1;
+        return k >= -60 && k <= 60;
+    }
+    std::string tmp2(std::ostringstream &o, const std::string &e, const std::string &ind)
+    {
+        std::string t = var();
+        o << ind << "const F2 " << t << " = " << e << ";\n";
+        return t;
+    }
+    // v as an F2 expression at exponent e
+    std::string at(std::ostringstream &o, const Val &v, int e, const std::string &ind)
+    {
+        if (v.isc) return lit2(v.c, e);
+        if (v.e == e) return v.x;
+        return tmp2(o, "kf2_mul1(" + fconst(std::ldexp(1.0, v.e - e)) + ", " + v.x + ")", ind);
+    }
+    Val emit2e(std::ostringstream &o, const Op &op, const std::vector<Val> &loads, const std::string &ind)
+    {
+        std::vector<Node> nodes;
+        std::vector<int> st;
+        for (const Instr &in : op.prog) {
+            Node n{in.op, in.arg, in.imm, {}};
+            int arity = 0;
+            switch (in.op) {
+            case KF_OP_LOAD: case KF_OP_CONST: arity = 0; break;
+            case KF_OP_ABS: case KF_OP_NEG: case KF_OP_SQRT: case KF_OP_EXP: case KF_OP_LOG: arity = 1; break;
+            case KF_OP_CLAMP: arity = 3; break;
+            case KF_OP_SELECT_GT: arity = 4; break;
+            case KF_OP_SHR: case KF_OP_SHL: case KF_OP_SAT_U8: case KF_OP_LUT:
+                fail(KF_ERR_PROGRAM, "codegen: integer opcode in a float program");
+            default: arity = 2;
+            }
+            n.ch.assign(st.end() - arity, st.end());
+            st.resize(st.size() - arity);
+            nodes.push_back(n);
+            st.push_back((int)nodes.size() - 1);
+        }
+        auto mk = [&](const std::string &e, int ex) { Val v; v.x = tmp2(o, e, ind); v.e = ex; return v; };
+        std::function<Val(int)> ev = [&](int i) -> Val {
+            const Node &n = nodes[i];
+            if (n.op == KF_OP_LOAD) return loads[op.kind == LOCAL ? 0 : n.arg];
+            if (n.op == KF_OP_CONST) { Val v; v.isc = true; v.c = (double)(float)n.imm; return v; }
+            if (n.op == KF_OP_ADD || n.op == KF_OP_SUB) {
+                const bool add = n.op == KF_OP_ADD;
+                const int a = n.ch[0], b = n.ch[1];
+                // a MUL child contracts into one FFMA2 (as emit2)
+                const int mi = nodes[b].op == KF_OP_MUL ? b : nodes[a].op == KF_OP_MUL ? a : -1;
+                if (mi >= 0) {
+                    Val m0 = ev(nodes[mi].ch[0]), m1 = ev(nodes[mi].ch[1]);
+                    Val x = ev(mi == b ? a : b);
+                    if (!(m0.isc && m1.isc)) {
+                        int ep;
+                        std::string f0, f1;
+                        if (m0.isc) { ep = m1.e; f0 = lit2(m0.c, 0); f1 = m1.x; }
+                        else if (m1.isc) { ep = m0.e; f0 = m0.x; f1 = lit2(m1.c, 0); }
+                        else { ep = m0.e + m1.e; f0 = m0.x; f1 = m1.x; }
+                        if (x.isc || !m0.isc || !m1.isc) {
+                            const std::string xs = at(o, x, ep, ind);
+                            const char *fn = mi == b ? (add ? "kf2_fma(" : "kf2_nfma(") : (add ? "kf2_fma(" : "kf2_fms(");
+                            return mk(std::string(fn) + f0 + ", " + f1 + ", " + xs + ")", ep);
+                        }
+                    }
+                    // fall through: both multiplicands constant
+                }
+                Val va = ev(a), vb = ev(b);
+                if (va.isc && vb.isc) {
+                    Val v;
+                    v.x = tmp2(o, std::string(add ? "kf2_add(" : "kf2_sub(") + lit2(va.c, 0) + ", " + lit2(vb.c, 0) + ")", ind);
+                    return v;
+                }
+                const int e = va.isc ? vb.e : va.e;
+                return mk(std::string(add ? "kf2_add(" : "kf2_sub(") + at(o, va, e, ind) + ", " + at(o, vb, e, ind) + ")", e);
+            }
+            if (n.op == KF_OP_MUL) {
+                Val va = ev(n.ch[0]), vb = ev(n.ch[1]);
+                int k = 0;
+                if (va.isc && vb.isc) return mk("kf2_mul(" + lit2(va.c, 0) + ", " + lit2(vb.c, 0) + ")", 0);
+                if (va.isc || vb.isc) {
+                    const Val &c = va.isc ? va : vb, &x = va.isc ? vb : va;
+                    if (pow2(c.c, k)) { Val r = x; r.e = x.e + k; return r; }   // free: the exponent moves
+                    return mk("kf2_mul1(" + fconst(c.c) + ", " + x.x + ")", x.e);
+                }
+                return mk("kf2_mul(" + va.x + ", " + vb.x + ")", va.e + vb.e);
+            }
+            if (n.op == KF_OP_DIV) {
+                Val va = ev(n.ch[0]), vb = ev(n.ch[1]);
+                int k = 0;
+                if (!va.isc && vb.isc && pow2(vb.c, k)) { Val r = va; r.e = va.e - k; return r; }
+                if (va.isc && vb.isc) return mk("kf2_div(" + lit2(va.c, 0) + ", " + lit2(vb.c, 0) + ")", 0);
+                if (vb.isc) return mk("kf2_div(" + va.x + ", " + lit2(vb.c, 0) + ")", va.e);
+                if (va.isc) return mk("kf2_div(" + lit2(va.c, vb.e) + ", " + vb.x + ")", 0);   // c / (s 2^e) = (c 2^-e / s) 2^0
+                return mk("kf2_div(" + va.x + ", " + vb.x + ")", va.e - vb.e);
+            }
+            if (n.op == KF_OP_MIN || n.op == KF_OP_MAX) {
+                Val va = ev(n.ch[0]), vb = ev(n.ch[1]);
+                const int e = va.isc ? vb.e : va.e;
+                const char *fn = n.op == KF_OP_MIN ? "kf2_min(" : "kf2_max(";
+                return mk(std::string(fn) + at(o, va, e, ind) + ", " + at(o, vb, e, ind) + ")", va.isc && vb.isc ? 0 : e);
+            }
+            if (n.op == KF_OP_ABS || n.op == KF_OP_NEG) {
+                Val va = ev(n.ch[0]);
+                const char *fn = n.op == KF_OP_ABS ? "kf2_abs(" : "kf2_neg(";
+                return mk(std::string(fn) + at(o, va, va.isc ? 0 : va.e, ind) + ")", va.isc ? 0 : va.e);
+            }
+            if (n.op == KF_OP_SQRT) {
+                Val va = ev(n.ch[0]);
+                const int e = va.isc ? 0 : (va.e % 2 == 0 ? va.e : va.e - 1);
+                return mk("kf2_sqrt(" + at(o, va, e, ind) + ")", e / 2);
+            }
+            if (n.op == KF_OP_CLAMP) {
+                Val vx = ev(n.ch[0]), vl = ev(n.ch[1]), vh = ev(n.ch[2]);
+                const int e = vx.isc ? 0 : vx.e;
+                return mk("kf2_clamp(" + at(o, vx, e, ind) + ", " + at(o, vl, e, ind) + ", " + at(o, vh, e, ind) + ")", e);
+            }
+            if (n.op == KF_OP_SELECT_GT) {
+                Val va = ev(n.ch[0]), vb = ev(n.ch[1]), vc = ev(n.ch[2]), vd = ev(n.ch[3]);
+                const int ec = va.isc ? vb.e : va.e, er = vc.isc ? vd.e : vc.e;
+                return mk("kf2_sel_gt(" + at(o, va, ec, ind) + ", " + at(o, vb, ec, ind) + ", " + at(o, vc, er, ind) + ", " +
+                              at(o, vd, er, ind) + ")", vc.isc && vd.isc ? 0 : er);
+            }
+            // EXP, LOG, POW: on true values
+            static const std::map<int, const char *> fn = {{KF_OP_EXP, "kf2_exp("}, {KF_OP_LOG, "kf2_log("}, {KF_OP_POW, "kf2_pow("}};
+            auto it = fn.find(n.op);
+            if (it == fn.end()) fail(KF_ERR_PROGRAM, "codegen: bad opcode");
+            std::string e = it->second;
+            for (size_t c = 0; c < n.ch.size(); c++) e += (c ? ", " : "") + at(o, ev(n.ch[c]), 0, ind);
+            return mk(e + ")", 0);
+        };
+        Val r = ev(st.back());
+        if (r.isc) { Val v; v.x = tmp2(o, lit2(r.c, 0), ind); return v; }
+        return r;
+    }
 };
 
 // ======================================================================= SWAR
@@ -753,6 +905,15 @@ struct StreamGen {
     std::map<std::tuple<int, int, int>, std::string> val_memo;
     std::map<std::tuple<std::string, int, int>, std::string> shfl_memo;   // (var, lane offset, edge key)
     std::map<std::tuple<int, int, int>, SwReg> sw_memo;                     // SWAR values (image, slot, column)
+    std::map<int, int> xe;   // pair mode: deferred power-of-two exponent of each image's stored values
+    int xe_of(int img) const { auto it = xe.find(img); return pm && it != xe.end() ? it->second : 0; }
+    void set_xe(int img, int e)
+    {
+        auto it = xe.find(img);
+        if (it != xe.end() && it->second != e) fail(KF_ERR_PROGRAM, "codegen: inconsistent deferred exponent");
+        xe[img] = e;
+    }
+    std::string cvalx(const Op &op, int e) const { return f32 ? fconst(std::ldexp((double)(float)op.constant, -e)) : cval(op); }
     std::map<std::tuple<std::string, int, int>, SwReg> swsh_memo;          // SWAR shuffles
     // variant being emitted
     int dir = 1;
@@ -760,6 +921,7 @@ struct StreamGen {
     bool pm = false;   // f32 values kept as packed pixel pairs (F2) for column-local math
     bool runptr = false;   // steady-state loop uses running row pointers (set per variant)
     bool vedge = false;    // variant starts at an image edge (peeled iterations remap taps)
+    bool defer_ok = true;  // pair mode: defer normalised masks' power-of-two scales (KFUSE_DEFER)
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
@@ -1117,10 +1279,16 @@ struct StreamGen {
         if (pm && op.kind == POINT) {
             const int ws = sl(img, 0, j);
             for (int q = 0; q < V / 2; q++) {
-                std::vector<std::string> loads;
-                for (int in : op.inputs) loads.push_back(pval(in, sl(in, HY(img) - HY(in), j), q));
-                const std::string r = pe.emit2(o, op, loads, ind);
-                o << ind << ring(img, ws, q) << " = " << r << ";\n";
+                std::vector<ProgEmitter::Val> loads;
+                for (int in : op.inputs) {
+                    ProgEmitter::Val v;
+                    v.x = pval(in, sl(in, HY(img) - HY(in), j), q);
+                    v.e = xe_of(in);
+                    loads.push_back(v);
+                }
+                const ProgEmitter::Val r = pe.emit2e(o, op, loads, ind);
+                set_xe(img, r.e);
+                o << ind << ring(img, ws, q) << " = " << r.x << ";\n";
             }
             return;
         }
@@ -1144,6 +1312,13 @@ struct StreamGen {
             auto mrow = [&](int dyp) { return ry + dir * dyp; };
             std::vector<std::string> acc(V);
             const Separable &sp = si.sep.at(k);
+            // pair mode: integer column weights, the mask's power-of-two scale deferred
+            const int ein = xe_of(in);
+            int ks = 0;
+            const bool defer = pm && defer_ok && sp.ok && ProgEmitter::pow2(sp.scale, ks);
+            if (!defer) ks = 0;
+            const double csc = defer ? sp.scale : 1.0;
+            const int eacc = ein + ks;
             if (sp.ok) {
                 // vertical pass in the lane's own columns, then horizontal taps
                 std::vector<std::pair<double, std::vector<std::string>>> rows;
@@ -1151,7 +1326,7 @@ struct StreamGen {
                 std::vector<double> cterms;   // coefficients of constant (exterior) rows
                 for (int dy = -ry; dy <= ry; dy++) {   // mask-row order in both directions (same rounding)
                     const int dyp = dir * dy;
-                    const double c = sp.col[mrow(dyp)];
+                    const double c = sp.col[mrow(dyp)] / csc;
                     if (c == 0.0) continue;
                     bool isc = false;
                     auto r = tap_row(img, op, in, dyp, j, u, isc, ind);
@@ -1165,7 +1340,7 @@ struct StreamGen {
                     for (double c : cterms) cs += c;
                     cst = var();
                     o << ind << "const " << KV() << " " << cst << " = kf_mul1(" << (f32 ? fconst(cs) : iconst((long long)cs))
-                      << ", " << cval(op) << ");\n";
+                      << ", " << cvalx(op, ein) << ");\n";
                 }
                 if (pm) {
                     for (int q = 0; q < V / 2; q++) {
@@ -1188,10 +1363,10 @@ struct StreamGen {
                 std::string csub;
                 if (op.mode == KF_CONSTANT && (el || er)) {
                     double cs = 0.0;
-                    for (double c : sp.col) cs += c;
+                    for (double c : sp.col) cs += c / csc;
                     csub = var();
                     o << ind << "const " << KV() << " " << csub << " = kf_mul1("
-                      << (f32 ? fconst(cs) : iconst((long long)cs)) << ", " << cval(op) << ");\n";
+                      << (f32 ? fconst(cs) : iconst((long long)cs)) << ", " << cvalx(op, ein) << ");\n";
                 }
                 for (int v = 0; v < V; v++) {
                     std::vector<std::pair<double, std::string>> terms;
@@ -1214,7 +1389,7 @@ struct StreamGen {
                         double m = op.mask[(size_t)mr * op.mw + dx + rx];
                         if (m == 0.0) continue;
                         for (int v = 0; v < V; v++)
-                            terms[v].push_back({m, isc ? cval(op) : at_col(row, v + dx, op, cval(op), ind)});
+                            terms[v].push_back({m, isc ? cvalx(op, ein) : at_col(row, v + dx, op, cvalx(op, ein), ind)});
                     }
                 }
                 for (int v = 0; v < V; v++) acc[v] = lincomb(terms[v], ind);
@@ -1222,9 +1397,12 @@ struct StreamGen {
             if (pm) {
                 const int ws = sl(img, 0, j);
                 for (int q = 0; q < V / 2; q++) {
-                    std::string pr = "make_float2(" + acc[2 * q] + ", " + acc[2 * q + 1] + ")";
-                    if (!op.prog.empty()) pr = pe.emit2(o, op, std::vector<std::string>{pr}, ind);
-                    o << ind << ring(img, ws, q) << " = " << pr << ";\n";
+                    ProgEmitter::Val a;
+                    a.x = "make_float2(" + acc[2 * q] + ", " + acc[2 * q + 1] + ")";
+                    a.e = eacc;
+                    if (!op.prog.empty()) a = pe.emit2e(o, op, std::vector<ProgEmitter::Val>{a}, ind);
+                    set_xe(img, a.e);
+                    o << ind << ring(img, ws, q) << " = " << a.x << ";\n";
                 }
                 return;
             }
@@ -1334,7 +1512,7 @@ struct StreamGen {
     // One iteration (slot j).  u >= 0: peeled edge iteration with index u.
     void iteration(int j, int u, const std::string &uexpr, const std::string &ind)
     {
-        const int P = si.P, D = si.D, L = si.L;
+        const int D = si.D, L = si.L;
         val_memo.clear();
         shfl_memo.clear();
         sw_memo.clear();
@@ -1366,6 +1544,21 @@ struct StreamGen {
         const int ss = sl(simg, 0, j);
         const bool store = !(u >= 0 && u < 2 * L);   // warm-up iterations store nothing
         std::string orow;   // output row pointer expression
+        // pair mode: the sink's deferred power-of-two exponent is applied here, once
+        std::vector<std::string> sk(V);
+        if (store && f32 && pm) {
+            const int e = xe_of(simg);
+            for (int q = 0; q < V / 2; q++) {
+                std::string pr = ring(simg, ss, q);
+                if (e != 0) {
+                    pr = var();
+                    o << ind << "const F2 " << pr << " = kf2_mul1(" << fconst(std::ldexp(1.0, e)) << ", " << ring(simg, ss, q)
+                      << ");\n";
+                }
+                sk[2 * q] = pr + ".x";
+                sk[2 * q + 1] = pr + ".y";
+            }
+        }
         if (!store) {
             o << ind << "{\n";
         } else if (runptr) {
@@ -1380,14 +1573,14 @@ struct StreamGen {
         if (!store) {
         } else if (!si.vec) {
             for (int v = 0; v < V; v++) {
-                std::string val = f32 ? (pm ? value(simg, ss, v, ind) : ring(simg, ss, v))
+                std::string val = f32 ? (pm ? sk[v] : ring(simg, ss, v))
                                       : si.swk.count(b.sink) ? ring(simg, ss, v)
                                                              : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
                 o << ind << "    if (x + " << v << " < a.fx1) (" << orow << ")[" << v << "] = " << val << ";\n";
             }
         } else if (f32) {
             o << ind << "    kf_st4f(" << orow;
-            for (int v = 0; v < V; v++) o << ", " << (pm ? value(simg, ss, v, ind) : ring(simg, ss, v));
+            for (int v = 0; v < V; v++) o << ", " << (pm ? sk[v] : ring(simg, ss, v));
             o << ");\n";
         } else {
             o << ind << "    kf_st4u(" << orow;
@@ -1527,6 +1720,7 @@ struct StreamGen {
     {
         for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
         pm = f32 && env_int("KFUSE_PAIRS", 1, 0, 1);
+        defer_ok = env_int("KFUSE_DEFER", 1, 0, 1);
 
         // Variants (the variant is CTA-uniform):
         //   interior strip, interior chunk   -- the hot loop, no border logic
@@ -1616,6 +1810,7 @@ static Separable factor(const Op &op, bool integer)
         for (auto &r : row) r = -r;
     }
     s.ok = true;
+    s.scale = scale;
     // the power-of-two scale goes to the column factor: the vertical pass runs
     // on packed pixel pairs, the horizontal one per pixel, so the horizontal
     // pass keeps its unit coefficients (one multiply fewer per pixel)

@@ -131,6 +131,7 @@ constexpr int kFrameTiles[2][2] = {{32, 8}, {8, 32}};    // frame tile shapes (w
 struct Separable {                // rank-1 mask: m[j][i] = col[j] * row[i]
     bool ok = false;
     std::vector<double> col, row;
+    double scale = 1.0;           // power-of-two factor folded into col (col / scale are integers)
 };
 
 // Interior streaming schedule of one block (codegen.cpp StreamGen)

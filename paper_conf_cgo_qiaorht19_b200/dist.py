@@ -126,3 +126,125 @@ def run_band(plan, band: Band, inputs, outputs, stream=None) -> None:
     """inputs: device tensors holding rows [in0, in1) (halo exchanged);
     outputs: device tensors of band.rows rows."""
     plan.run_band(band.row0, band.row1, inputs, band.in0, band.in1, outputs, stream)
+
+
+# ---------------------------------------------------------------------------
+# Halo rows over peer memory (NVLink P2P through CUDA IPC mappings): the north
+# star's "read from peer memory over NVLink" path.  No host collective per
+# step: three stream-ordered kernels of libkfuse (kf_peer_signal / _pull /
+# _wait) synchronise through monotonic device counters, so a whole step --
+# signal, core rows, halo pull, edge strips -- is plain launches on ONE stream
+# and can be captured into a CUDA graph.  The exchange latency hides behind
+# the core rows: a neighbour's signal is issued before its own core kernel.
+
+# counter slots (uint32) of each rank
+_READY_ABOVE, _READY_BELOW, _SEEN_ABOVE, _SEEN_BELOW, _ACK_ABOVE, _ACK_BELOW, _SENT, _ERR = range(8)
+
+
+class PeerHalo:
+    """Maps the neighbours' input buffers and counters into this process
+    (torch.multiprocessing's CUDA IPC reductions, exchanged once with
+    all_gather_object) and runs the band steps over them.
+
+    bufs: this rank's rotating input buffers, each holding rows [in0, in1) of
+    the global image (first dim = rows).  Every rank must pass the same number
+    of buffers, and call step() the same number of times with the same set
+    indices, in the same order."""
+
+    def __init__(self, band: Band, bufs, group=None, spin_limit: int = 1 << 27):
+        from torch.multiprocessing.reductions import reduce_tensor
+        self.band, self.bufs, self.spin = band, list(bufs), spin_limit
+        self.ctr = torch.zeros(8, dtype=torch.int32, device=self.bufs[0].device)
+        mine = {"ctr": reduce_tensor(self.ctr), "bufs": [reduce_tensor(b) for b in self.bufs],
+                "top": band.top, "rows": band.rows}
+        every = [None] * band.world
+        dist.all_gather_object(every, mine, group=group)
+
+        def open_(red):
+            fn, args = red
+            return fn(*args)
+
+        def peer(r):
+            d = every[r]
+            return {"ctr": open_(d["ctr"]), "bufs": [open_(x) for x in d["bufs"]], "top": d["top"], "rows": d["rows"]}
+
+        self.up = peer(band.rank - 1) if band.rank > 0 and band.top > 0 else None
+        self.down = peer(band.rank + 1) if band.rank < band.world - 1 and band.bottom > 0 else None
+
+    def _c(self, slot: int, ctr=None) -> int:
+        return (self.ctr if ctr is None else ctr).data_ptr() + 4 * slot
+
+    def errors(self) -> int:
+        """Non-zero when a wait timed out (a neighbour never signalled)."""
+        return int(self.ctr[_ERR].item())
+
+    def signal(self, stream) -> None:
+        """This step's own rows are ready (everything queued before on `stream`)."""
+        from . import kfuse as K
+        flags = []
+        if self.up:
+            flags.append(self._c(_READY_BELOW, self.up["ctr"]))
+        if self.down:
+            flags.append(self._c(_READY_ABOVE, self.down["ctr"]))
+        K.peer_signal(flags, self._c(_SENT), stream)
+
+    def pull(self, s: int, stream) -> None:
+        """Copies the neighbours' boundary rows of buffer set s into the halo rows."""
+        from . import kfuse as K
+        b, buf = self.band, self.bufs[s]
+        rb = buf[0].numel() * buf.element_size()
+        dst, src, nb, flag, seen, ack = [], [], [], [], [], []
+        if self.up:
+            u = self.up
+            dst.append(buf.data_ptr())
+            src.append(u["bufs"][s].data_ptr() + (u["top"] + u["rows"] - b.top) * rb)
+            nb.append(b.top * rb)
+            flag.append(self._c(_READY_ABOVE))
+            seen.append(self._c(_SEEN_ABOVE))
+            ack.append(self._c(_ACK_BELOW, u["ctr"]))
+        if self.down:
+            d = self.down
+            dst.append(buf.data_ptr() + (b.top + b.rows) * rb)
+            src.append(d["bufs"][s].data_ptr() + d["top"] * rb)
+            nb.append(b.bottom * rb)
+            flag.append(self._c(_READY_BELOW))
+            seen.append(self._c(_SEEN_BELOW))
+            ack.append(self._c(_ACK_ABOVE, d["ctr"]))
+        K.peer_pull(dst, src, nb, flag, seen, ack, self._c(_ERR), self.spin, stream)
+
+    def wait_consumed(self, stream) -> None:
+        """Before the own rows are overwritten: both neighbours pulled every step signalled."""
+        from . import kfuse as K
+        cnt = ([self._c(_ACK_ABOVE)] if self.up else []) + ([self._c(_ACK_BELOW)] if self.down else [])
+        K.peer_wait(cnt, [self._c(_SENT)] * len(cnt), self._c(_ERR), self.spin, stream)
+
+    def step(self, plan, s: int, outputs, stream, side=None) -> None:
+        """One band step on buffer set s: core rows on `stream` while `side`
+        (a second stream, forked from `stream`) signals and pulls the halo rows;
+        then the edge strips on `stream`.  Bit-identical to exchange_halos +
+        run_band.  With side=None everything runs on `stream`, in the order
+        signal, core, pull, edges.  Without neighbours it is just the core."""
+        b = self.band
+        (c0, c1), edges = split_rows(b)
+        ins = [self.bufs[s]]
+        exch = self.up is not None or self.down is not None
+        if exch and side is not None:
+            side.wait_stream(stream)          # the own rows of this step are ready
+            self.signal(side)
+            self.pull(s, side)
+        elif exch:
+            self.signal(stream)
+        if c1 > c0:
+            plan.run_band(c0, c1, ins, b.in0, b.in1, [o[c0 - b.row0:c1 - b.row0] for o in outputs], stream)
+        if exch and side is not None:
+            stream.wait_stream(side)
+        elif exch:
+            self.pull(s, stream)
+        for r0, r1 in edges:
+            plan.run_band(r0, r1, ins, b.in0, b.in1, [o[r0 - b.row0:r1 - b.row0] for o in outputs], stream)
+
+    def close(self) -> None:
+        """Drops the peer mappings.  Call on every rank (synchronised) before any
+        rank frees the buffers it exported."""
+        self.up = self.down = None
+        torch.cuda.synchronize()

@@ -65,6 +65,9 @@ _SIGS = {
     "kf_mark_output": (C.c_int, [_P, C.c_int32]),
     "kf_plan_fusion": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
     "kf_plan_basic": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
+    "kf_peer_signal": (C.c_int, [_P, C.c_int32, _P, _P]),
+    "kf_peer_pull": (C.c_int, [C.c_int32, _P, _P, _P, _P, _P, _P, _P, C.c_int64, _P]),
+    "kf_peer_wait": (C.c_int, [C.c_int32, _P, _P, _P, C.c_int64, _P]),
     "kf_plan_exact": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
     "kf_plan_unfused": (C.c_int, [_P, C.POINTER(_P)]),
     "kf_plan_from_blocks": (C.c_int, [_P, _I32P, C.POINTER(_P)]),
@@ -314,6 +317,27 @@ def _stream(stream) -> int:
     if isinstance(stream, int):
         return stream
     return stream.cuda_stream
+
+
+def _i64s(vals) -> C.Array:
+    return (C.c_int64 * max(1, len(vals)))(*[int(v) for v in vals])
+
+
+def peer_signal(flags, sent=0, stream=None) -> None:
+    """kf_peer_signal: release-increment counters (device addresses, may be peer)."""
+    _check(lib.kf_peer_signal(_ptrs(flags), len(flags), _P(int(sent)), _P(_stream(stream))))
+
+
+def peer_pull(dst, src, nbytes, flag, seen, ack, err, spin_limit=1 << 27, stream=None) -> None:
+    """kf_peer_pull over len(dst) segments (all arguments device addresses; ack entries may be 0)."""
+    _check(lib.kf_peer_pull(len(dst), _ptrs(dst), _ptrs(src), _i64s(nbytes), _ptrs(flag), _ptrs(seen),
+                            _ptrs(ack), _P(int(err)), int(spin_limit), _P(_stream(stream))))
+
+
+def peer_wait(counter, target, err, spin_limit=1 << 27, stream=None) -> None:
+    """kf_peer_wait: wait until every counter[i] reaches target[i] (device addresses)."""
+    _check(lib.kf_peer_wait(len(counter), _ptrs(counter), _ptrs(target), _P(int(err)), int(spin_limit),
+                            _P(_stream(stream))))
 
 
 def version() -> str:

@@ -298,3 +298,95 @@ def test_c5_full_size_and_four_bands():
         torch.cuda.synchronize()
         assert torch.equal(b_out, full[band.row0:band.row1]), f"band {r} differs"
         del b_in, b_out
+
+
+# ------------------------------------------- halo rows over peer memory (§8(e))
+
+
+def _peer_worker(rank, world, port, wl, graph, q):
+    import os as _os
+    import torch.distributed as dist
+    from paper_conf_cgo_qiaorht19_b200 import dist as KD
+    _os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)   # one GPU: the ranks share it, the IPC path is the same as across GPUs
+        spec = P.WORKLOADS[wl](96, 130)
+        W, H = spec["width"], spec["height"]
+        plan = make_plan(spec, "b200")
+        band = KD.partition(H, world, rank, plan.halo_rows)
+        imgs = [gen.image(spec["dtype"], 40 + k, W, H) for k in range(3)]
+        fulls = [run_gpu(spec, plan, [im])[0] for im in imgs]
+
+        def own(k):   # a buffer with this band's own rows of image k, halo rows poisoned
+            t = torch.from_numpy(np.ascontiguousarray(imgs[k][band.in0:band.in1])).cuda()
+            t[:band.top] = 77
+            t[band.top + band.rows:] = 77
+            return t
+
+        bufs = [own(0), own(1)]
+        halo = KD.PeerHalo(band, bufs, spin_limit=1 << 24)
+        side = torch.cuda.Stream() if graph else None
+        outs = [torch.empty((band.rows,) + fulls[0].shape[1:], dtype=bufs[0].dtype, device="cuda") for _ in bufs]
+        s = torch.cuda.Stream()
+        ok = True
+        if graph:
+            for k in (0, 1):
+                halo.step(plan, k, [outs[k]], s, side)   # warm-up (also outside the graph)
+            s.synchronize()
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=s):
+                for k in (0, 1):
+                    halo.step(plan, k, [outs[k]], s, side)
+            for _ in range(3):
+                with torch.cuda.stream(s):
+                    g.replay()
+        else:
+            for it in range(4):
+                halo.step(plan, it % 2, [outs[it % 2]], s)
+        s.synchronize()
+        for k in (0, 1):
+            ok &= bool(np.array_equal(outs[k].cpu().numpy(), fulls[k][band.row0:band.row1]))
+        # overwrite set 0 with image 2 once both neighbours consumed it, then run again
+        halo.wait_consumed(s)
+        with torch.cuda.stream(s):
+            bufs[0][band.top:band.top + band.rows].copy_(own(2)[band.top:band.top + band.rows])
+        halo.step(plan, 0, [outs[0]], s)
+        s.synchronize()
+        ok &= bool(np.array_equal(outs[0].cpu().numpy(), fulls[2][band.row0:band.row1]))
+        q.put((rank, ok, halo.errors()))
+        halo.close()          # every rank drops its peer mappings before anyone frees
+        dist.barrier()
+        del halo, bufs, outs
+        torch.cuda.synchronize()
+        dist.barrier()
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("wl,world,graph", [("harris", 2, False), ("harris", 3, True), ("deep10", 2, True)])
+def test_peer_halo_steps(wl, world, graph):
+    """dist.PeerHalo: halo rows pulled from the neighbours' buffers through CUDA
+    IPC mappings, synchronised by device counters (kf_peer_signal / _pull / _wait),
+    eager and captured in a CUDA graph, with rotating buffer sets and an
+    overwrite guarded by wait_consumed -- bit-identical to the full-image run.
+    The ranks share one GPU here; across GPUs the same mappings are NVLink peers."""
+    import socket
+    import torch.multiprocessing as mp
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_peer_worker, args=(r, world, port, wl, graph, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in procs:
+        r, ok, err = q.get(timeout=300)
+        res[r] = (ok, err)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    assert all(ok and err == 0 for ok, err in res.values()), res
