@@ -138,9 +138,13 @@ __device__ __forceinline__ I4 kf_mac(I4 acc, int m, I4 v)
 }
 
 // -------------------------------------------------------------- float
-__device__ __forceinline__ float kf_add(float a, float b) { return a + b; }
-__device__ __forceinline__ float kf_sub(float a, float b) { return a - b; }
-__device__ __forceinline__ float kf_mul(float a, float b) { return a * b; }
+// Explicitly rounded forms: the compiler never contracts a product into a
+// later addition, so every code variant of a fused kernel (edge strips, peeled
+// warm-up iterations, steady-state loop) rounds the same operations the same
+// way and band / strip decompositions stay bit-identical.
+__device__ __forceinline__ float kf_add(float a, float b) { return __fadd_rn(a, b); }
+__device__ __forceinline__ float kf_sub(float a, float b) { return __fsub_rn(a, b); }
+__device__ __forceinline__ float kf_mul(float a, float b) { return __fmul_rn(a, b); }
 __device__ __forceinline__ float kf_div(float a, float b) { return a / b; }
 __device__ __forceinline__ float kf_min(float a, float b) { return fminf(a, b); }
 __device__ __forceinline__ float kf_max(float a, float b) { return fmaxf(a, b); }
@@ -197,23 +201,42 @@ __device__ __forceinline__ I4 kf_shdn(I4 v, int d)
               __shfl_down_sync(KF_FULL, v.z, d), __shfl_down_sync(KF_FULL, v.w, d)};
 }
 // first product of an accumulation (mask coefficient m)
-__device__ __forceinline__ float kf_mul1(float m, float v) { return m * v; }
+__device__ __forceinline__ float kf_mul1(float m, float v) { return __fmul_rn(m, v); }
 __device__ __forceinline__ I4 kf_mul1(int m, I4 v) { return I4{m * v.x, m * v.y, m * v.z, m * v.w}; }
 
 // ------------------------------------------------ packed f32x2 (sm_100a)
 // Two adjacent pixels of a lane as one 64-bit register pair: FFMA2 / FADD2 /
 // FMUL2 issue one instruction for both.  Operations without a
 // packed form run per component.
+//
+// ptxas contracts a packed FMUL2 into a following FADD2 (one FFMA2, one
+// rounding) even for mul.rn/add.rn.f32x2, and only where the product has a
+// single use -- so the same expression rounded differently in the peeled
+// warm-up iterations than in the loop (measured: band runs differed from the
+// whole-image run by a few ulps).  A packed product whose rounding matters is
+// therefore an FFMA2 with an addend of -0.0 the compiler cannot see
+// (a * b + (-0) == a * b exactly, signed zeros included): there is no multiply
+// left to contract.  Multiplies by a power of two are exact and stay FMUL2.
 typedef float2 F2;
+#ifdef KF_NVRTC
+__constant__ float kf_nz = -0.0f;   // never written; opaque to the compiler
+#define KF_NZ2 make_float2(kf_nz, kf_nz)
+#else
+#define KF_NZ2 make_float2(-0.0f, -0.0f)
+#endif
+__device__ __forceinline__ bool kf_pow2f(float m) { return (__float_as_uint(m) & 0x007fffffu) == 0u && m != 0.0f; }
 __device__ __forceinline__ F2 kf2(float a) { return make_float2(a, a); }
 __device__ __forceinline__ F2 kf2_add(F2 a, F2 b) { return __fadd2_rn(a, b); }
 __device__ __forceinline__ F2 kf2_sub(F2 a, F2 b) { return __fadd2_rn(a, make_float2(-b.x, -b.y)); }
-__device__ __forceinline__ F2 kf2_mul(F2 a, F2 b) { return __fmul2_rn(a, b); }
+__device__ __forceinline__ F2 kf2_mul(F2 a, F2 b) { return __ffma2_rn(a, b, KF_NZ2); }
 __device__ __forceinline__ F2 kf2_fma(F2 a, F2 b, F2 c) { return __ffma2_rn(a, b, c); }          // a*b + c
 __device__ __forceinline__ F2 kf2_fms(F2 a, F2 b, F2 c) { return __ffma2_rn(a, b, make_float2(-c.x, -c.y)); }  // a*b - c
 __device__ __forceinline__ F2 kf2_nfma(F2 a, F2 b, F2 c) { return __ffma2_rn(make_float2(-a.x, -a.y), b, c); }  // c - a*b
 __device__ __forceinline__ F2 kf2_mac(F2 acc, float m, F2 v) { return __ffma2_rn(v, make_float2(m, m), acc); }
-__device__ __forceinline__ F2 kf2_mul1(float m, F2 v) { return __fmul2_rn(v, make_float2(m, m)); }
+__device__ __forceinline__ F2 kf2_mul1(float m, F2 v)
+{
+    return kf_pow2f(m) ? __fmul2_rn(v, make_float2(m, m)) : __ffma2_rn(v, make_float2(m, m), KF_NZ2);
+}
 __device__ __forceinline__ F2 kf2_div(F2 a, F2 b) { return make_float2(a.x / b.x, a.y / b.y); }
 __device__ __forceinline__ F2 kf2_min(F2 a, F2 b) { return make_float2(fminf(a.x, b.x), fminf(a.y, b.y)); }
 __device__ __forceinline__ F2 kf2_max(F2 a, F2 b) { return make_float2(fmaxf(a.x, b.x), fmaxf(a.y, b.y)); }
