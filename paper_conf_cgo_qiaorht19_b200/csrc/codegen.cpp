@@ -922,6 +922,7 @@ struct StreamGen {
     bool runptr = false;   // steady-state loop uses running row pointers (set per variant)
     bool vedge = false;    // variant starts at an image edge (peeled iterations remap taps)
     bool defer_ok = true;  // pair mode: defer normalised masks' power-of-two scales (KFUSE_DEFER)
+    std::set<int> prp;     // external images fed by running row pointers from the prologue on (interior strips)
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
@@ -1479,7 +1480,7 @@ struct StreamGen {
     void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
     {
         int s = slot.at(img);
-        if (runptr) {   // steady state: running row pointer (rows stay inside [base, rlast])
+        if (runptr || prp.count(img)) {   // running row pointer (rows stay inside [base, rlast])
             o << ind << "if ((" << it << ") < nit) kf_cp16(sr" << s << " + (" << ss << ") * 32, ip" << s << ");\n";
             o << ind << "ip" << s << " += dW;\n";
             return;
@@ -1493,7 +1494,10 @@ struct StreamGen {
     {
         int s = slot.at(img);
         std::string q = var();
-        o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = sr" << s << "[(" << ss << ") * 32];\n";
+        if (si.lpf)   // the row was read from the ring one iteration ago
+            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = pf" << s << ";\n";
+        else
+            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = sr" << s << "[(" << ss << ") * 32];\n";
         if (pm) {
             o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
             o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
@@ -1530,8 +1534,18 @@ struct StreamGen {
             }
             for (int img : b.ext) issue(img, s_iss, uexpr + " + " + std::to_string(j + DS - 1), ind);
             o << ind << "kf_cp_commit();\n";
-            o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
-            for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
+            if (si.lpf) {
+                // this iteration's row is already in registers; wait for the next
+                // row and read it now, a whole iteration before its use
+                for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
+                const std::string s_nxt = u >= 0 ? std::to_string((u + 1) % DS)
+                                                 : (j + 1 < si.P && !si.rolled ? "qb + " + std::to_string(j + 1) : "qnext");
+                o << ind << "kf_cp_wait<" << DS - 2 << ">();\n";
+                for (int img : b.ext) o << ind << "pf" << slot.at(img) << " = sr" << slot.at(img) << "[(" << s_nxt << ") * 32];\n";
+            } else {
+                o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
+                for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
+            }
         } else {
             for (int img : b.ext) load(img, sl(img, D, j), uexpr + " + " + std::to_string(j + D), ind);
         }
@@ -1652,6 +1666,22 @@ struct StreamGen {
                 }
             o << ";\n";
         }
+        // Interior strips (downward, not at an image edge) read rows
+        // [ys - L, ye + L) of an image needed with the full halo L, which the
+        // launch geometry keeps inside [base, rlast]: no clamps, one running
+        // pointer from the first prologue row on.
+        prp.clear();
+        if (si.sring && !ve && dir > 0 && env_int("KFUSE_PRO_RP", 1, 0, 1))
+            for (int img : b.ext)
+                if (HY(img) == L) prp.insert(img);
+        if (!prp.empty()) {
+            o << "    const int dW = W;\n";
+            for (int img : prp) {
+                int s = slot.at(img);
+                o << "    const " << RT() << " *__restrict__ ip" << s << " = g" << s << " + (ys - " << 2 * L - HY(img)
+                  << ") * W;\n";
+            }
+        }
         if (si.sring) {
             for (int img : b.ext) {
                 int s = slot.at(img);
@@ -1661,6 +1691,13 @@ struct StreamGen {
             for (int it = 0; it < si.DS - 1; it++) {
                 for (int img : b.ext) issue(img, std::to_string(it), std::to_string(it), "    ");
                 o << "    kf_cp_commit();\n";
+            }
+            if (si.lpf) {
+                o << "    kf_cp_wait<" << si.DS - 2 << ">();\n";
+                for (int img : b.ext) {
+                    int s = slot.at(img);
+                    o << "    " << (f32 ? "float4" : "uint4") << " pf" << s << " = sr" << s << "[0];\n";
+                }
             }
             o << "    int qb = 0;   // ring slot of the current iteration's row (multiple of the unroll)\n";
         } else {
@@ -1691,8 +1728,9 @@ struct StreamGen {
         // fetches after the prologue lies inside [base, rlast])
         const bool rp_ok = si.sring && si.DS - 1 >= 2 * L;
         if (rp_ok) {
-            o << "    const int dW = " << (dir > 0 ? "W" : "-W") << ";\n";
+            if (prp.empty()) o << "    const int dW = " << (dir > 0 ? "W" : "-W") << ";\n";
             for (int img : b.ext) {
+                if (prp.count(img)) continue;   // already positioned at row u0 + DS - 1
                 int s = slot.at(img);
                 std::string row = row_of(img, std::to_string(u0 + si.DS - 1), "    ");
                 o << "    const " << RT() << " *__restrict__ ip" << s << " = g" << s << " + " << row << " * W;\n";
@@ -1705,10 +1743,12 @@ struct StreamGen {
             o << "    #pragma unroll 1\n";
             o << "    for (int u = " << u0 << "; u < nit; u++) {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
+            if (si.lpf) o << "        const int qnext = qb + 1 == " << si.DS << " ? 0 : qb + 1;\n";
             iteration(0, -1, "u", "        ");
         } else {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
+            if (si.lpf) o << "        const int qnext = qb + " << P << " == " << si.DS << " ? 0 : qb + " << P << ";\n";
             for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
         }
         if (si.sring) o << "        qb += " << step << ";\n        if (qb == " << si.DS << ") qb = 0;\n";
@@ -1889,6 +1929,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         if (DS > cap || DS < 2) si.sring = false;
         si.DS = DS;
         si.ring_bytes = (int)b.ext.size() * DS * 512;
+        si.lpf = si.sring && DS >= 3 && env_int("KFUSE_LDS_PF", 1, 0, 1);
     }
     if (!si.sring) si.P = std::max(maxdepth, maxdepth_ext + si.D);
     // register estimate: live ring values (depth per image, D prefetched rows)

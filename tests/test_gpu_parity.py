@@ -390,3 +390,16 @@ def test_peer_halo_steps(wl, world, graph):
         p.join(timeout=120)
         assert p.exitcode == 0
     assert all(ok and err == 0 for ok, err in res.values()), res
+
+
+@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "deep10"])
+def test_strip_geometry_bit_identical(wl, monkeypatch):
+    """The fused result does not depend on how the interior is cut into strips
+    (peeled warm-up iterations vs the steady-state loop round identically)."""
+    spec = P.WORKLOADS[wl](256, 240)
+    ins = _inputs(spec, 9)
+    plan = make_plan(spec, "b200")
+    base = run_gpu(spec, plan, ins)[0]
+    for ns in (2, 5, 40, 118):
+        monkeypatch.setenv("KFUSE_NSTRIPS", str(ns))
+        np.testing.assert_array_equal(run_gpu(spec, plan, ins)[0], base)
