@@ -1775,7 +1775,18 @@ struct StreamGen {
             variant(-1, true, si.edge_l, si.edge_r);
         }
         o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast(const KfArgs &a, const int item)\n{\n";
-        o << "    const int chunk = item % a.n_chunks, strip = item / a.n_chunks;\n";
+        if (env_int("KFUSE_HEAVY_FIRST", 1, 0, 1)) {
+            // heavy items first: the edge strips (longer peeled prologues) and the
+            // edge chunks (lane selects) start in the first wave instead of
+            // forming the tail of the last one
+            o << "    const int s0 = item / a.n_chunks, c0 = item % a.n_chunks;\n";
+            o << "    const int strip = a.edge_b ? (a.edge_t ? (s0 == 0 ? 0 : s0 == 1 ? a.n_strips - 1 : s0 - 1)\n"
+                 "                                      : (s0 == 0 ? a.n_strips - 1 : s0 - 1)) : s0;\n";
+            o << "    const int chunk = a.edge_r ? (a.edge_l ? (c0 == 0 ? 0 : c0 == 1 ? a.n_chunks - 1 : c0 - 1)\n"
+                 "                                      : (c0 == 0 ? a.n_chunks - 1 : c0 - 1)) : c0;\n";
+        } else {
+            o << "    const int chunk = item % a.n_chunks, strip = item / a.n_chunks;\n";
+        }
         if (si.edge_v) {
             o << "    if (a.edge_t && strip == 0) { " << kernel_name(block) << "_fast" << vname(1, true, si.edge_l, si.edge_r)
               << "(a, chunk, strip); return; }\n";
@@ -1879,7 +1890,7 @@ static int prog_size(const Op &op)
         case KF_OP_POW: n += 80; break;
         case KF_OP_LOG: n += 30; break;
         case KF_OP_EXP: n += 25; break;
-        case KF_OP_SQRT: n += 8; break;
+        case KF_OP_SQRT: n += 2; break;   // MUFU.SQRT (kf_sqrt)
         case KF_OP_DIV: n += 15; break;
         default: n += 1;
         }
