@@ -265,6 +265,13 @@ def bench_single(args, cfg_name, spec, seed) -> None:
                 "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
                 "peak_source": peaks["source"],
                 "per_launch": f"{ab} B/px x {px} px = {ab * px} algorithmic bytes per launch"}
+    # Same-size memory floor: the framework's own 1-in/1-out copy kernel (same
+    # launch path, streaming loop and buffer rotation) over the same pixel count.
+    # Context for `frac`: at these sizes the ramp and drain of a ~20 us kernel
+    # keep even a copy below the large-transfer copy peak.
+    if not args.no_extra:
+        roofline["copy_floor"] = copy_floor(W, H, ins, stream, torch, ab * px)
+        roofline["copy_floor"]["fused_over_copy"] = round(roofline["copy_floor"]["ms_per_step"] / head["ms_per_step"], 4)
     # end to end through the public API with host buffers (pinned)
     e2e_steps = max(3, min(args.steps, 20))
     hin = torch.from_numpy(host).pin_memory()
@@ -298,6 +305,24 @@ def bench_single(args, cfg_name, spec, seed) -> None:
         "workloads": extra,
     }
     print(json.dumps(out))
+
+
+def copy_floor(W, H, ins, stream, torch, fused_bytes) -> dict:
+    """Times the `copy` diagnostic pipeline (one point kernel, out = in, 8 B/px)
+    over W x H f32 pixels, exactly like the fused plan (graph replay, rotating
+    buffer sets larger than L2).  A u8x4 image has the same 4 B/px."""
+    from kf_inputs import pipelines as P
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+    n = len(ins)
+    cin = [torch.empty((H, W), dtype=torch.float32, device="cuda").uniform_() for _ in range(n)]
+    cout = [torch.empty_like(x) for x in cin]
+    plan = K.Pipeline.from_spec(P.copy(W, H)).plan_fusion("b200")
+    plan.prepare()
+    ms = time_plan(plan, cin, cout, 200, 3, stream, torch)
+    del cin, cout
+    gbs = 8 * W * H / (ms * 1e-3) / 1e9
+    return {"ms_per_step": round(ms, 5), "gbs": round(gbs, 1), "frac_of_peak": round(gbs / load_peaks()["hbm_gbs"], 4),
+            "what": "the framework's own copy kernel (8 B/px) over the same pixel count"}
 
 
 def bench_extra(args, stream, torch, clocks) -> dict:
@@ -337,6 +362,9 @@ def bench_extra(args, stream, torch, clocks) -> dict:
                                 "hbm_frac": round(ab * px / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4) if ab else None}
         f = d["plans"]["b200"]
         d["fused_vs_unfused"] = round(d["plans"]["unfused"]["ms_per_step"] / f["ms_per_step"], 3)
+        if px >= 1 << 22:
+            d["copy_floor"] = copy_floor(W, H, ins, stream, torch, 8 * px)
+            d["copy_floor"]["fused_over_copy"] = round(d["copy_floor"]["ms_per_step"] / f["ms_per_step"], 4)
         ipp = ncu_inst(cfg, "b200")
         if ipp:
             issue = ipp * px / (f["ms_per_step"] * 1e-3)

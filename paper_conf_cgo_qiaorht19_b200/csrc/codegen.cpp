@@ -468,9 +468,14 @@ struct SwEmitter {
         if (o) {
             r.lo = var();
             r.hi = var();
-            const std::string m = lit(0xffff >> n);
-            *o << ind << "const unsigned " << r.lo << " = (" << a.lo << " >> " << n << ") & " << m << ";\n";
-            *o << ind << "const unsigned " << r.hi << " = (" << a.hi << " >> " << n << ") & " << m << ";\n";
+            if (n == 8) {   // each lane's high byte moved down: one PRMT instead of SHF + LOP3 (both ALU pipe)
+                *o << ind << "const unsigned " << r.lo << " = __byte_perm(" << a.lo << ", 0u, 0x4341);\n";
+                *o << ind << "const unsigned " << r.hi << " = __byte_perm(" << a.hi << ", 0u, 0x4341);\n";
+            } else {
+                const std::string m = lit(0xffff >> n);
+                *o << ind << "const unsigned " << r.lo << " = (" << a.lo << " >> " << n << ") & " << m << ";\n";
+                *o << ind << "const unsigned " << r.hi << " = (" << a.hi << " >> " << n << ") & " << m << ";\n";
+            }
         }
         return r;
     }
@@ -923,6 +928,7 @@ struct StreamGen {
     bool vedge = false;    // variant starts at an image edge (peeled iterations remap taps)
     bool defer_ok = true;  // pair mode: defer normalised masks' power-of-two scales (KFUSE_DEFER)
     std::set<int> prp;     // external images fed by running row pointers from the prologue on (interior strips)
+    bool qptr = false;     // steady-state loop: ring slots addressed from per-trip base pointers
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
@@ -1477,17 +1483,28 @@ struct StreamGen {
         return row;
     }
     // shared-memory ring: start the copy of iteration `it`'s row into ring slot `ss`
+    // Address of ring slot `ss` of image slot s.  In the steady-state loop the
+    // slots are addressed from per-trip base pointers (sq = slot qb, sp = qprev,
+    // sn = qnext) so that the unrolled rows use immediate offsets.
+    std::string slot_ptr(int s, const std::string &ss) const
+    {
+        if (qptr) {
+            if (ss == "qprev") return "sp" + std::to_string(s);
+            if (ss == "qnext") return "sn" + std::to_string(s);
+            if (ss.rfind("qb + ", 0) == 0) return "sq" + std::to_string(s) + " + " + std::to_string(32 * std::stoi(ss.substr(5)));
+        }
+        return "sr" + std::to_string(s) + " + (" + ss + ") * 32";
+    }
     void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
     {
         int s = slot.at(img);
         if (runptr || prp.count(img)) {   // running row pointer (rows stay inside [base, rlast])
-            o << ind << "if ((" << it << ") < nit) kf_cp16(sr" << s << " + (" << ss << ") * 32, ip" << s << ");\n";
+            o << ind << "if ((" << it << ") < nit) kf_cp16(" << slot_ptr(s, ss) << ", ip" << s << ");\n";
             o << ind << "ip" << s << " += dW;\n";
             return;
         }
         std::string row = row_of(img, it, ind);
-        o << ind << "if ((" << it << ") < nit) kf_cp16(sr" << s << " + (" << ss << ") * 32, g" << s << " + " << row
-          << " * W);\n";
+        o << ind << "if ((" << it << ") < nit) kf_cp16(" << slot_ptr(s, ss) << ", g" << s << " + " << row << " * W);\n";
     }
     // shared-memory ring: read ring slot `ss` into register ring slot rs
     void fetch(int img, const std::string &ss, int rs, const std::string &ind)
@@ -1497,7 +1514,7 @@ struct StreamGen {
         if (si.lpf)   // the row was read from the ring one iteration ago
             o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = pf" << s << ";\n";
         else
-            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = sr" << s << "[(" << ss << ") * 32];\n";
+            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = *(" << slot_ptr(s, ss) << ");\n";
         if (pm) {
             o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
             o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
@@ -1541,7 +1558,7 @@ struct StreamGen {
                 const std::string s_nxt = u >= 0 ? std::to_string((u + 1) % DS)
                                                  : (j + 1 < si.P && !si.rolled ? "qb + " + std::to_string(j + 1) : "qnext");
                 o << ind << "kf_cp_wait<" << DS - 2 << ">();\n";
-                for (int img : b.ext) o << ind << "pf" << slot.at(img) << " = sr" << slot.at(img) << "[(" << s_nxt << ") * 32];\n";
+                for (int img : b.ext) o << ind << "pf" << slot.at(img) << " = *(" << slot_ptr(slot.at(img), s_nxt) << ");\n";
             } else {
                 o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
                 for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
@@ -1629,7 +1646,12 @@ struct StreamGen {
         o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast" << vname(dir, ve, l, r)
           << "(const KfArgs &a, const int chunk, const int strip)\n{\n";
         o << "    const int lane = threadIdx.x & 31;\n";
-        o << "    const int W = a.W, H = a.H;\n    (void)H;\n";
+        // The image size is fixed per pipeline (one iteration space):
+        // baked in, row strides become immediates and unrolled rows use address offsets.
+        if (env_int("KFUSE_CONST_W", 1, 0, 1))
+            o << "    constexpr int W = " << p->W << ", H = " << p->H << ";\n    (void)H;\n";
+        else
+            o << "    const int W = a.W, H = a.H;\n    (void)H;\n";
         o << "    const int x = a.fx0 + (chunk * " << 32 - 2 * HL << " + lane - " << HL << ") * " << V << ";\n";
         o << "    const bool xst = lane >= " << HL << " && lane < " << 32 - HL << " && x < a.fx1;\n";
         // strip bounds in primed (streaming-direction) rows
@@ -1749,7 +1771,17 @@ struct StreamGen {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
             if (si.lpf) o << "        const int qnext = qb + " << P << " == " << si.DS << " ? 0 : qb + " << P << ";\n";
+            qptr = si.sring && env_int("KFUSE_QPTR", 1, 0, 1);
+            if (qptr)
+                for (int img : b.ext) {
+                    const int s = slot.at(img);
+                    const char *T = f32 ? "float4" : "uint4";
+                    o << "        " << T << " *const sq" << s << " = sr" << s << " + qb * 32;\n";
+                    o << "        " << T << " *const sp" << s << " = sr" << s << " + qprev * 32;\n";
+                    if (si.lpf) o << "        " << T << " *const sn" << s << " = sr" << s << " + qnext * 32;\n";
+                }
             for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
+            qptr = false;
         }
         if (si.sring) o << "        qb += " << step << ";\n        if (qb == " << si.DS << ") qb = 0;\n";
         o << "    }\n}\n\n";
