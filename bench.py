@@ -254,6 +254,12 @@ def bench_single(args, cfg_name, spec, seed) -> None:
                          "launches": plan.num_launches, "alg_bytes_per_px": ab,
                          "alg_gbs": round(ab * px / (ms * 1e-3) / 1e9, 1) if ab else None}
     head = results[args.plan]
+    # distribution over repeated timed replays (the paper reports the median of
+    # 500 runs): 11 replays of min(K, 100) steps each, ms/step
+    if not args.no_extra:
+        reps = sorted(time_plan(plans[args.plan][1], ins, outs, min(args.steps, 100), 1, stream, torch) for _ in range(11))
+        head["replays"] = {"n": 11, "steps_each": min(args.steps, 100), "median_ms": round(reps[5], 5),
+                           "min_ms": round(reps[0], 5), "iqr_ms": round(reps[8] - reps[2], 5)}
     peaks = load_peaks()
     _, hplan = plans[args.plan]
     ab = head["alg_bytes_per_px"] or 8
