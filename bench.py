@@ -291,6 +291,8 @@ def bench_single(args, cfg_name, spec, seed) -> None:
     e2e_s = (time.perf_counter() - t) / e2e_steps
     e2e = {"value": round(px / e2e_s / 1e6, 1), "unit": UNIT, "h2d_bytes_per_step": int(hin.numel() * hin.element_size()),
            "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps}
+    if not args.no_extra:
+        e2e["pcie_floor"] = pcie_floor(hin, hout, px, torch)
     # CPU baseline: the unfused oracle on this box's host, one full image
     cpu = None
     if not args.no_cpu:
@@ -311,6 +313,31 @@ def bench_single(args, cfg_name, spec, seed) -> None:
         "workloads": extra,
     }
     print(json.dumps(out))
+
+
+def pcie_floor(hin, hout, px, torch) -> dict:
+    """The e2e leg's ceiling on this box: the same H2D and D2H byte counts as one
+    step, copied concurrently on two streams with no kernel in between (what
+    kf_run_host overlaps with its row bands).  Wall time over 5 repetitions."""
+    d_in = torch.empty(hin.shape, dtype=hin.dtype, device="cuda")
+    d_out = torch.empty(hout.shape, dtype=hout.dtype, device="cuda")
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+
+    def both():
+        with torch.cuda.stream(s1):
+            d_in.copy_(hin, non_blocking=True)
+        with torch.cuda.stream(s2):
+            hout.copy_(d_out, non_blocking=True)
+        torch.cuda.synchronize()
+    both()
+    t = time.perf_counter()
+    for _ in range(5):
+        both()
+    dt = (time.perf_counter() - t) / 5
+    nb = hin.numel() * hin.element_size() + hout.numel() * hout.element_size()
+    del d_in, d_out
+    return {"value": round(px / dt / 1e6, 1), "unit": UNIT, "gbs_both_directions": round(nb / dt / 1e9, 1),
+            "what": "H2D + D2H of one step's bytes, concurrent, no compute: the ceiling of e2e"}
 
 
 def copy_floor(W, H, ins, stream, torch, fused_bytes) -> dict:
