@@ -1738,7 +1738,7 @@ struct StreamGen {
                 if (p->ops[k].kind == LOCAL)
                     need = std::max(need, 2 * L - HY(p->n_inputs + k) + p->ops[k].ry());
         if (need > 0) {
-            const int Q = (need + P - 1) / P * P;
+            const int Q = si.rolled ? need : (need + P - 1) / P * P;
             for (int u = 0; u < Q; u++) iteration(u % P, u, std::to_string(u - u % P), "      ");
             u0 = Q;
             if (si.sring) o << "    qb = " << Q % si.DS << ";\n";
@@ -2044,7 +2044,10 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     // left to the frame path
     const long long budget = env_int("KFUSE_CODE_BUDGET", 12000, 0, 1 << 30);
     si.rolled = ops * si.P * 6 > budget;
-    if (si.rolled) si.edge_v = false;
+    // rolled bodies keep the edge strips too (peeled remapped prologue, then
+    // the rolled loop), unless KFUSE_ROLLED_EDGE_V=0 leaves those rows to the
+    // frame: for deep10 the frame's index-exchange tiles cost 12 % of the kernel
+    if (si.rolled && !env_int("KFUSE_ROLLED_EDGE_V", 1, 0, 1)) si.edge_v = false;
     si.edge_l = !rep && hfit && p->W >= 4 * kStreamV;
     si.edge_r = si.edge_l && si.vec;
     si.ok = b.Rx <= 2 * kStreamV * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
