@@ -2040,8 +2040,8 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     }
     si.edge_v = !rep && p->H >= 4 * si.L + 2 * si.P + 8;
     // unrolled: ~P copies per variant (4 variants + 2 peeled prologues); too
-    // much straight-line code for NVRTC/ptxas -> rolled body, vertical edges
-    // left to the frame path
+    // much straight-line code for NVRTC/ptxas and the instruction cache ->
+    // one rolled body copy
     const long long budget = env_int("KFUSE_CODE_BUDGET", 12000, 0, 1 << 30);
     si.rolled = ops * si.P * 6 > budget;
     // rolled bodies keep the edge strips too (peeled remapped prologue, then

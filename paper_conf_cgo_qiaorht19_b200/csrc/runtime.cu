@@ -451,8 +451,17 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     KF_CUDA(cudaStreamWaitEvent(rt.s_h2d, rt.ev_start, 0));
     KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_start, 0));
     int copied = 0;   // input rows [0, copied) are queued on the H2D stream
+    // Band boundaries.  Only the first band's upload and the last band's
+    // download are exposed (everything else overlaps), so with 8 bands the
+    // ends are thin: row shares 1,3,6,6,6,6,3,1 / 32 (uniform when fewer bands).
+    static const int kShare8[9] = {0, 1, 4, 10, 16, 22, 28, 31, 32};
+    auto cut = [&](int k) {
+        if (nb == kHostBands && kHostBands == 8 && env_int("KFUSE_HOST_TAPER", 1, 0, 1))
+            return (int)((long long)p->H * kShare8[k] / 32);
+        return (int)((long long)p->H * k / nb);
+    };
     for (int k = 0; k < nb; k++) {
-        const int r0 = (int)((long long)p->H * k / nb), r1 = (int)((long long)p->H * (k + 1) / nb);
+        const int r0 = cut(k), r1 = cut(k + 1);
         const int need = k == nb - 1 ? p->H : std::min(p->H, r1 + R);
         if (need > copied) {
             for (int i = 0; i < n_in; i++)
