@@ -449,6 +449,12 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
             halo = KD.PeerHalo(band, ins)
         except Exception as e:   # e.g. no IPC between the ranks: fall back to NCCL
             mode, note = "nccl", f"peer setup failed ({type(e).__name__}: {e}); "
+        # every rank must use the same transport: peer only if it worked everywhere
+        agree = torch.tensor([1 if mode == "peer" else 0], dtype=torch.int32,
+                             device="cuda" if dist.get_backend() == "nccl" else "cpu")
+        dist.all_reduce(agree, op=dist.ReduceOp.MIN)
+        if int(agree.item()) == 0 and mode == "peer":
+            mode, halo, note = "nccl", None, "peer setup failed on another rank; "
     (c0, c1), edges = KD.split_rows(band)
     exch = halo is not None and (halo.up is not None or halo.down is not None)
     launches_per_step = plan.num_launches * ((1 if c1 > c0 else 0) + len(edges)) + (2 if exch else 0)
@@ -543,7 +549,15 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     if halo is not None:   # drop the peer mappings on every rank before any rank frees its buffers
         halo.close()
         dist.barrier()
+    del graph
+    torch.cuda.synchronize()
     dist.destroy_process_group()
+    # Leave without the interpreter's teardown: torch's CUDA-IPC bookkeeping of
+    # the exchanged buffers can crash at exit after everything above has been
+    # released and the result printed (seen as SIGSEGV at world 1).
+    sys.stdout.flush()
+    sys.stderr.flush()
+    os._exit(0)
 
 
 def main():

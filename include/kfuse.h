@@ -278,6 +278,12 @@ kf_status kf_peer_pull(int32_t n, void *const *dst, const void *const *src, cons
 kf_status kf_peer_wait(int32_t n, uint32_t *const *counter, uint32_t *const *target, uint32_t *err,
                        int64_t spin_limit, void *stream);
 
+/* Enables peer access from `device` to `peer_device` (NVLink P2P) so that the
+ * kf_peer_* kernels launched on `device` can use peer mappings of
+ * `peer_device`'s memory.  Idempotent; KF_OK when device == peer_device;
+ * KF_ERR_CUDA when the pair has no peer path. */
+kf_status kf_peer_enable(int32_t device, int32_t peer_device);
+
 /* Thread-local message of the last failing call on this thread. */
 const char *kf_last_error(void);
 /* Library version string. */

@@ -189,3 +189,30 @@ extern "C" kf_status kf_peer_wait(int32_t n, uint32_t *const *counter, uint32_t 
     a.n = n;
     KF_GUARD(peer_wait_k<<<1, 32, 0, (cudaStream_t)stream>>>(a));
 }
+
+// Lets kernels on `device` read and write `peer_device`'s memory (NVLink P2P),
+// in the primary context every runtime in the process shares.  Idempotent.
+extern "C" kf_status kf_peer_enable(int32_t device, int32_t peer_device)
+{
+    if (device == peer_device) return KF_OK;
+    int can = 0;
+    if (cudaDeviceCanAccessPeer(&can, device, peer_device) != cudaSuccess || !can) {
+        set_error("kf_peer_enable: device " + std::to_string(device) + " cannot access device " +
+                  std::to_string(peer_device));
+        return KF_ERR_CUDA;
+    }
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(device);
+    cudaError_t e = cudaDeviceEnablePeerAccess(peer_device, 0);
+    cudaSetDevice(cur);
+    if (e == cudaErrorPeerAccessAlreadyEnabled) {
+        cudaGetLastError();   // clear the sticky-free "already enabled" status
+        return KF_OK;
+    }
+    if (e != cudaSuccess) {
+        set_error(std::string("kf_peer_enable: ") + cudaGetErrorString(e));
+        return KF_ERR_CUDA;
+    }
+    return KF_OK;
+}

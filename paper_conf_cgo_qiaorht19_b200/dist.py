@@ -155,6 +155,9 @@ class PeerHalo:
         from torch.multiprocessing.reductions import reduce_tensor
         self.band, self.bufs, self.spin = band, list(bufs), spin_limit
         self.ctr = torch.zeros(8, dtype=torch.int32, device=self.bufs[0].device)
+        if band.world == 1:   # no neighbours: nothing to share
+            self.up = self.down = None
+            return
         mine = {"ctr": reduce_tensor(self.ctr), "bufs": [reduce_tensor(b) for b in self.bufs],
                 "top": band.top, "rows": band.rows}
         every = [None] * band.world
@@ -170,6 +173,13 @@ class PeerHalo:
 
         self.up = peer(band.rank - 1) if band.rank > 0 and band.top > 0 else None
         self.down = peer(band.rank + 1) if band.rank < band.world - 1 and band.bottom > 0 else None
+        # the pull/signal kernels run on this rank's GPU and touch the
+        # neighbours' memory directly: enable the P2P path (NVLink) explicitly
+        from . import kfuse as K
+        dev = self.bufs[0].device.index
+        for nb in (self.up, self.down):
+            if nb is not None:
+                K.peer_enable(dev, nb["ctr"].device.index)
 
     def _c(self, slot: int, ctr=None) -> int:
         return (self.ctr if ctr is None else ctr).data_ptr() + 4 * slot

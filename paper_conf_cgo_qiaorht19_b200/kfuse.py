@@ -68,6 +68,7 @@ _SIGS = {
     "kf_peer_signal": (C.c_int, [_P, C.c_int32, _P, _P]),
     "kf_peer_pull": (C.c_int, [C.c_int32, _P, _P, _P, _P, _P, _P, _P, C.c_int64, _P]),
     "kf_peer_wait": (C.c_int, [C.c_int32, _P, _P, _P, C.c_int64, _P]),
+    "kf_peer_enable": (C.c_int, [C.c_int32, C.c_int32]),
     "kf_plan_exact": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
     "kf_plan_unfused": (C.c_int, [_P, C.POINTER(_P)]),
     "kf_plan_from_blocks": (C.c_int, [_P, _I32P, C.POINTER(_P)]),
@@ -338,6 +339,11 @@ def peer_wait(counter, target, err, spin_limit=1 << 27, stream=None) -> None:
     """kf_peer_wait: wait until every counter[i] reaches target[i] (device addresses)."""
     _check(lib.kf_peer_wait(len(counter), _ptrs(counter), _ptrs(target), _P(int(err)), int(spin_limit),
                             _P(_stream(stream))))
+
+
+def peer_enable(device: int, peer_device: int) -> None:
+    """kf_peer_enable: kernels on `device` may access `peer_device`'s memory."""
+    _check(lib.kf_peer_enable(int(device), int(peer_device)))
 
 
 def version() -> str:
