@@ -424,6 +424,18 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     rank, world = dist.get_rank(), dist.get_world_size()
     dev = int(os.environ.get("KFUSE_BENCH_DEVICE", os.environ.get("LOCAL_RANK", rank)))
     torch.cuda.set_device(dev)
+    # NCCL prints its version banner on stdout when the first communicator is
+    # created: create it now with stdout pointed at stderr (stdout carries the
+    # one JSON line)
+    sys.stdout.flush()
+    saved = os.dup(1)
+    os.dup2(2, 1)
+    try:
+        dist.barrier()
+    finally:
+        sys.stdout.flush()
+        os.dup2(saved, 1)
+        os.close(saved)
     W, Hb = spec["width"], spec["height"]
     Htot = Hb * world                                 # weak scaling: one band per GPU
     gspec = P.WORKLOADS[spec["name"]](W, Htot)
