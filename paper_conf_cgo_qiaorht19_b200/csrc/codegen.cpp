@@ -2090,11 +2090,18 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     }
     o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << env_int("KFUSE_MINCTAS", kMinCtasPerSm, 1, 32) << ") " << kernel_name(b, block)
       << "(const __grid_constant__ KfArgs a)\n{\n";
-    o << "    const int cta = blockIdx.x;\n";
-    o << "    if (cta < a.frame_ctas) { " << kernel_name(block) << "_frame(a, cta); return; }\n";
-    // one warp per CTA: the item index and the trip count are CTA-uniform, so
-    // the warp shuffles of the interior path need no convergence barriers
-    if (si.ok) o << "    " << kernel_name(block) << "_fast(a, cta - a.frame_ctas);\n";
+    // Persistent CTAs: the grid is at most one wave of resident CTAs, and each
+    // loops over work items (frame tiles first, then interior items) with a
+    // grid stride -- no per-item CTA launch.  One warp per CTA: the item index
+    // and the trip count are CTA-uniform, so the warp shuffles of the interior
+    // path need no convergence barriers.  No cp.async copy is in flight between
+    // items (every issued row was waited for), so the shared ring is reused.
+    o << "    const int total = a.frame_ctas + a.n_items;\n";
+    o << "    for (int cta = blockIdx.x; cta < total; cta += gridDim.x) {\n";
+    o << "        if (cta < a.frame_ctas) " << kernel_name(block) << "_frame(a, cta);\n";
+    if (si.ok) o << "        else " << kernel_name(block) << "_fast(a, cta - a.frame_ctas);\n";
+    o << "        __syncwarp();\n";
+    o << "    }\n";
     o << "}\n";
     return o.str();
 }

@@ -391,10 +391,20 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         a.r1 = bhi[bi];
         if (a.r1 <= a.r0) continue;
         unsigned grid = launch_geometry(a, b, cb);
+        if (!cb.si.ok) a.n_items = 0;   // frame-only block
         if (const char *skip = getenv("KFUSE_DIAG_SKIP")) {   // timing diagnostics only: wrong results
             if (!strcmp(skip, "frame")) { grid -= a.frame_ctas; a.frame_ctas = 0; a.n_rect = 0; }
-            if (!strcmp(skip, "fast")) { grid = a.frame_ctas; }
+            if (!strcmp(skip, "fast")) { grid = a.frame_ctas; a.n_items = 0; }
         }
+        {   // Optional persistent CTAs (KFUSE_PERSIST=1): at most one wave, the kernel
+            // strides over the items.  Off by default: measured slower (C3 27.4 ->
+            // 30.0 us, C4 327 -> 363; profiles/r01_sweep_persist.jsonl) -- the
+            // hardware refilling freed CTA slots balances better than a static stride.
+            const long long slots = (long long)cb.num_sms * cb.ctas_per_sm *
+                                    env_int("KFUSE_PERSIST_WAVES", 1, 1, 1 << 20);
+            if (env_int("KFUSE_PERSIST", 0, 0, 1) && (long long)grid > slots) grid = (unsigned)slots;
+        }
+        if (grid == 0) continue;
         void *params[] = {&a};
         cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
     }
