@@ -117,6 +117,18 @@ def test_argument_validation():
         K.Pipeline(0, 5, "f32")
 
 
+def test_peer_calls_validate_without_a_gpu():
+    """The multi-GPU entry points check their arguments before touching CUDA:
+    same-device peer enable is a no-op; bad segment counts fail with KF_ERR_ARG."""
+    K.peer_enable(0, 0)
+    with pytest.raises(K.KfError) as e:
+        K.peer_wait([1] * 5, [1] * 5, 8, stream=0)          # more than 4 counters
+    assert e.value.name == "KF_ERR_ARG"
+    with pytest.raises(K.KfError) as e:
+        K.peer_signal([1] * 5, stream=0)
+    assert e.value.name == "KF_ERR_ARG"
+
+
 def test_repeat_mixing_is_not_fused():
     """Reading R-8: a fused block's local kernels all use REPEAT or none does."""
     p = P.Pipeline("mix", 16, 16, "f32")
