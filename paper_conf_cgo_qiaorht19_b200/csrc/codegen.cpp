@@ -905,6 +905,8 @@ struct StreamGen {
     std::ostringstream &o;
     int tmp = 0;
     ProgEmitter pe;
+    const int V;      // pixels per lane (si.V)
+    const int NQ;     // float4 / uint4 vectors per lane per row (V / 4)
     std::map<int, int> slot;   // external image -> slot
     // per-iteration memo: (image, ring slot, column) -> unpacked value variable
     std::map<std::tuple<int, int, int>, std::string> val_memo;
@@ -931,11 +933,11 @@ struct StreamGen {
     bool qptr = false;     // steady-state loop: ring slots addressed from per-trip base pointers
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
-        : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
+        : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp},
+          V(si_.V), NQ(si_.V / 4)
     {
     }
 
-    static constexpr int V = kStreamV;
     std::string KV() const { return f32 ? "float" : "I4"; }
     std::string RT() const { return f32 ? "float" : "unsigned"; }   // ring storage type
     std::string var() { return "v" + std::to_string(tmp++); }
@@ -1030,7 +1032,7 @@ struct StreamGen {
                 sub = m < 0 ? csub : row[V - 1 - m];
             }
             std::string t2 = var();
-            o << ind << "const " << KV() << " " << t2 << " = (" << (q < 0 ? "x == 0" : "x == W - 4") << ") ? "
+            o << ind << "const " << KV() << " " << t2 << " = (" << (q < 0 ? "x == 0" : "x == W - " + std::to_string(V)) << ") ? "
               << sub << " : " << t << ";\n";
             t = t2;
         }
@@ -1183,7 +1185,7 @@ struct StreamGen {
                 slo = sr.lo;
                 shi = sr.hi;
             }
-            const std::string cond = q < 0 ? "x == 0" : "x == W - 4";
+            const std::string cond = q < 0 ? "x == 0" : "x == W - " + std::to_string(V);
             SwReg t2 = t;
             t2.lo = var();
             t2.hi = var();
@@ -1432,6 +1434,25 @@ struct StreamGen {
         }
     }
 
+    // ring slot rs of image img from the NQ 128-bit vectors q[0..NQ) of one row
+    // (pixel v is component v % 4 of vector v / 4)
+    void unpack_row(int img, int rs, const std::vector<std::string> &q, const std::string &ind)
+    {
+        const char *c[4] = {"x", "y", "z", "w"};
+        auto comp = [&](int v) { return q[v / 4] + "." + c[v % 4]; };
+        if (pm) {
+            for (int k = 0; k < V / 2; k++)
+                o << ind << ring(img, rs, k) << " = make_float2(" << comp(2 * k) << ", " << comp(2 * k + 1) << ");\n";
+        } else if (si.swring.count(img)) {
+            for (int v = 0; v < V; v++) {
+                o << ind << ring(img, rs, 2 * v) << " = __byte_perm(" << comp(v) << ", 0u, 0x4140);\n";
+                o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(" << comp(v) << ", 0u, 0x4342);\n";
+            }
+        } else {
+            for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << comp(v) << ";\n";
+        }
+    }
+
     // prefetch of external image `img` for iteration `it` into ring slot rs
     void load(int img, int rs, const std::string &it, const std::string &ind)
     {
@@ -1443,20 +1464,13 @@ struct StreamGen {
         std::string ptr = "g" + std::to_string(s) + " + " + row + " * W";
         const char *c[4] = {"x", "y", "z", "w"};
         if (si.vec) {
-            std::string q = var();
-            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = " << (f32 ? "kf_ld4f(" : "kf_ld4u(")
-              << ptr << ");\n";
-            if (pm) {
-                o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
-                o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
-            } else if (si.swring.count(img)) {
-                for (int v = 0; v < V; v++) {
-                    o << ind << ring(img, rs, 2 * v) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4140);\n";
-                    o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4342);\n";
-                }
-            } else {
-                for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
+            std::vector<std::string> q(NQ);
+            for (int k = 0; k < NQ; k++) {
+                q[k] = var();
+                o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q[k] << " = " << (f32 ? "kf_ld4f(" : "kf_ld4u(")
+                  << ptr << " + " << 4 * k << ");\n";
             }
+            unpack_row(img, rs, q, ind);
         } else if (pm) {
             for (int q = 0; q < V / 2; q++)
                 o << ind << ring(img, rs, q) << " = make_float2(__ldg(" << ptr << " + cl" << 2 * q << "), __ldg(" << ptr
@@ -1491,43 +1505,42 @@ struct StreamGen {
         if (qptr) {
             if (ss == "qprev") return "sp" + std::to_string(s);
             if (ss == "qnext") return "sn" + std::to_string(s);
-            if (ss.rfind("qb + ", 0) == 0) return "sq" + std::to_string(s) + " + " + std::to_string(32 * std::stoi(ss.substr(5)));
+            if (ss.rfind("qb + ", 0) == 0) return "sq" + std::to_string(s) + " + " + std::to_string(32 * NQ * std::stoi(ss.substr(5)));
         }
-        return "sr" + std::to_string(s) + " + (" + ss + ") * 32";
+        return "sr" + std::to_string(s) + " + (" + ss + ") * " + std::to_string(32 * NQ);
+    }
+    // the NQ 16-byte copies of one lane's row segment (lane-contiguous: a warp row is 512 * NQ bytes)
+    void cp_row(const std::string &dst, const std::string &src, const std::string &guard, const std::string &ind)
+    {
+        o << ind << "if (" << guard << ") {";
+        for (int k = 0; k < NQ; k++) o << " kf_cp16(" << dst << (k ? " + " + std::to_string(k) : "") << ", " << src
+                                       << (k ? " + " + std::to_string(4 * k) : "") << ");";
+        o << " }\n";
     }
     void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
     {
         int s = slot.at(img);
         if (runptr || prp.count(img)) {   // running row pointer (rows stay inside [base, rlast])
-            o << ind << "if ((" << it << ") < nit) kf_cp16(" << slot_ptr(s, ss) << ", ip" << s << ");\n";
+            cp_row(slot_ptr(s, ss), "ip" + std::to_string(s), "(" + it + ") < nit", ind);
             o << ind << "ip" << s << " += dW;\n";
             return;
         }
         std::string row = row_of(img, it, ind);
-        o << ind << "if ((" << it << ") < nit) kf_cp16(" << slot_ptr(s, ss) << ", g" << s << " + " << row << " * W);\n";
+        cp_row(slot_ptr(s, ss), "g" + std::to_string(s) + " + " + row + " * W", "(" + it + ") < nit", ind);
     }
     // shared-memory ring: read ring slot `ss` into register ring slot rs
     void fetch(int img, const std::string &ss, int rs, const std::string &ind)
     {
         int s = slot.at(img);
-        std::string q = var();
-        if (si.lpf)   // the row was read from the ring one iteration ago
-            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = pf" << s << ";\n";
-        else
-            o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q << " = *(" << slot_ptr(s, ss) << ");\n";
-        if (pm) {
-            o << ind << ring(img, rs, 0) << " = make_float2(" << q << ".x, " << q << ".y);\n";
-            o << ind << ring(img, rs, 1) << " = make_float2(" << q << ".z, " << q << ".w);\n";
-        } else if (si.swring.count(img)) {
-            const char *c[4] = {"x", "y", "z", "w"};
-            for (int v = 0; v < V; v++) {
-                o << ind << ring(img, rs, 2 * v) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4140);\n";
-                o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(" << q << "." << c[v] << ", 0u, 0x4342);\n";
-            }
-        } else {
-            const char *c[4] = {"x", "y", "z", "w"};
-            for (int v = 0; v < V; v++) o << ind << ring(img, rs, v) << " = " << q << "." << c[v] << ";\n";
+        std::vector<std::string> q(NQ);
+        for (int k = 0; k < NQ; k++) {
+            q[k] = var();
+            if (si.lpf)   // the row was read from the ring one iteration ago
+                o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q[k] << " = pf" << s << "_" << k << ";\n";
+            else
+                o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q[k] << " = *(" << slot_ptr(s, ss) << " + " << k << ");\n";
         }
+        unpack_row(img, rs, q, ind);
     }
 
     // One iteration (slot j).  u >= 0: peeled edge iteration with index u.
@@ -1558,7 +1571,9 @@ struct StreamGen {
                 const std::string s_nxt = u >= 0 ? std::to_string((u + 1) % DS)
                                                  : (j + 1 < si.P && !si.rolled ? "qb + " + std::to_string(j + 1) : "qnext");
                 o << ind << "kf_cp_wait<" << DS - 2 << ">();\n";
-                for (int img : b.ext) o << ind << "pf" << slot.at(img) << " = *(" << slot_ptr(slot.at(img), s_nxt) << ");\n";
+                for (int img : b.ext)
+                    for (int k = 0; k < NQ; k++)
+                        o << ind << "pf" << slot.at(img) << "_" << k << " = *(" << slot_ptr(slot.at(img), s_nxt) << " + " << k << ");\n";
             } else {
                 o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
                 for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
@@ -1610,14 +1625,18 @@ struct StreamGen {
                 o << ind << "    if (x + " << v << " < a.fx1) (" << orow << ")[" << v << "] = " << val << ";\n";
             }
         } else if (f32) {
-            o << ind << "    kf_st4f(" << orow;
-            for (int v = 0; v < V; v++) o << ", " << (pm ? sk[v] : ring(simg, ss, v));
-            o << ");\n";
+            for (int k = 0; k < NQ; k++) {
+                o << ind << "    kf_st4f(" << orow << (k ? " + " + std::to_string(4 * k) : "");
+                for (int v = 4 * k; v < 4 * k + 4; v++) o << ", " << (pm ? sk[v] : ring(simg, ss, v));
+                o << ");\n";
+            }
         } else {
-            o << ind << "    kf_st4u(" << orow;
-            for (int v = 0; v < V; v++)
-                o << ", " << (si.swk.count(b.sink) ? ring(simg, ss, v) : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")");
-            o << ");\n";
+            for (int k = 0; k < NQ; k++) {
+                o << ind << "    kf_st4u(" << orow << (k ? " + " + std::to_string(4 * k) : "");
+                for (int v = 4 * k; v < 4 * k + 4; v++)
+                    o << ", " << (si.swk.count(b.sink) ? ring(simg, ss, v) : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")");
+                o << ");\n";
+            }
         }
         o << ind << "}\n";
         if (runptr) o << ind << "op += dW;\n";
@@ -1708,7 +1727,7 @@ struct StreamGen {
             for (int img : b.ext) {
                 int s = slot.at(img);
                 o << "    " << (f32 ? "float4" : "uint4") << " *sr" << s << " = (" << (f32 ? "float4" : "uint4")
-                  << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 << ") + lane;\n";
+                  << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 * NQ << ") + lane * " << NQ << ";\n";
             }
             for (int it = 0; it < si.DS - 1; it++) {
                 for (int img : b.ext) issue(img, std::to_string(it), std::to_string(it), "    ");
@@ -1718,7 +1737,8 @@ struct StreamGen {
                 o << "    kf_cp_wait<" << si.DS - 2 << ">();\n";
                 for (int img : b.ext) {
                     int s = slot.at(img);
-                    o << "    " << (f32 ? "float4" : "uint4") << " pf" << s << " = sr" << s << "[0];\n";
+                    for (int k = 0; k < NQ; k++)
+                        o << "    " << (f32 ? "float4" : "uint4") << " pf" << s << "_" << k << " = sr" << s << "[" << k << "];\n";
                 }
             }
             o << "    int qb = 0;   // ring slot of the current iteration's row (multiple of the unroll)\n";
@@ -1776,9 +1796,9 @@ struct StreamGen {
                 for (int img : b.ext) {
                     const int s = slot.at(img);
                     const char *T = f32 ? "float4" : "uint4";
-                    o << "        " << T << " *const sq" << s << " = sr" << s << " + qb * 32;\n";
-                    o << "        " << T << " *const sp" << s << " = sr" << s << " + qprev * 32;\n";
-                    if (si.lpf) o << "        " << T << " *const sn" << s << " = sr" << s << " + qnext * 32;\n";
+                    o << "        " << T << " *const sq" << s << " = sr" << s << " + qb * " << 32 * NQ << ";\n";
+                    o << "        " << T << " *const sp" << s << " = sr" << s << " + qprev * " << 32 * NQ << ";\n";
+                    if (si.lpf) o << "        " << T << " *const sn" << s << " = sr" << s << " + qnext * " << 32 * NQ << ";\n";
                 }
             for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
             qptr = false;
@@ -1933,11 +1953,15 @@ static int prog_size(const Op &op)
 StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
 {
     StreamInfo si;
-    si.vec = p->W % kStreamV == 0;
+    // f32 blocks may run 8 pixels per lane (two float4 per row per lane):
+    // half the shuffles and per-row overhead per pixel, twice the ring registers
+    si.V = (p->dtype == KF_F32 && env_int("KFUSE_V8", 0, 0, 1)) ? 8 : kStreamV;
+    const int kV_ = si.V;
+    si.vec = p->W % kV_ == 0;
     for (int img : b.ext) si.hy[img] = b.ext_hy.at(img);
     for (int k : b.kernels) si.hy[p->n_inputs + k] = b.hy.at(k);
     si.L = b.Ry;
-    si.HL = std::max(1, (b.Rx + kStreamV - 1) / kStreamV);
+    si.HL = std::max(1, (b.Rx + kV_ - 1) / kV_);
     // history depth of every image, in iterations
     int maxdepth_ext = 1, maxdepth = 1;
     for (auto &kv : si.hy) si.depth[kv.first] = 1;
@@ -1965,13 +1989,13 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     if (si.sring) {
         si.P = std::max(maxdepth, maxdepth_ext);
         const int want = env_int("KFUSE_SMEM_ROWS", 12, 2, 64);
-        const int cap = 32768 / (512 * (int)b.ext.size());   // <= 32 KB of ring per warp
+        const int cap = 32768 / (128 * kV_ * (int)b.ext.size());   // <= 32 KB of ring per warp
         int DS = std::max(want, si.P + 1);
         DS = (DS + si.P - 1) / si.P * si.P;
         while (DS > cap && DS - si.P >= si.P + 1) DS -= si.P;
         if (DS > cap || DS < 2) si.sring = false;
         si.DS = DS;
-        si.ring_bytes = (int)b.ext.size() * DS * 512;
+        si.ring_bytes = (int)b.ext.size() * DS * 128 * kV_;
         si.lpf = si.sring && DS >= 3 && env_int("KFUSE_LDS_PF", 1, 0, 1);
     }
     if (!si.sring) si.P = std::max(maxdepth, maxdepth_ext + si.D);
@@ -1979,7 +2003,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     int live = 0;
     for (auto &kv : si.depth) {
         bool ext = std::binary_search(b.ext.begin(), b.ext.end(), kv.first);
-        live += (kv.second + (ext && !si.sring ? si.D : 0)) * kStreamV;
+        live += (kv.second + (ext && !si.sring ? si.D : 0)) * kV_;
     }
     // SWAR rings: a u8x4 image read at several rows per
     // iteration by SWAR local kernels keeps its ring unpacked -- (lo, hi) per
@@ -2003,7 +2027,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         }
         std::sort(cand.begin(), cand.end(), [](auto &a, auto &b2) { return a.first != b2.first ? a.first > b2.first : a.second < b2.second; });
         for (auto &c : cand) {
-            const int extra = c.first * kStreamV;
+            const int extra = c.first * kV_;
             if (live + extra > cap) continue;
             live += extra;
             si.swring.insert(c.second);
@@ -2022,9 +2046,9 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
             int taps = sp.ok ? (int)(std::count_if(sp.col.begin(), sp.col.end(), [](double c) { return c != 0.0; }) +
                                      std::count_if(sp.row.begin(), sp.row.end(), [](double c) { return c != 0.0; }))
                              : nnz;
-            ops += (long long)(taps + 2 * op.rx() + prog_size(op)) * kStreamV * ch;
+            ops += (long long)(taps + 2 * op.rx() + prog_size(op)) * kV_ * ch;
         } else {
-            ops += (long long)prog_size(op) * kStreamV * ch;
+            ops += (long long)prog_size(op) * kV_ * ch;
         }
     }
     si.iter_ops = ops;
@@ -2036,7 +2060,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         const Op &op = p->ops[k];
         if (op.kind != LOCAL) continue;
         rep |= op.mode == KF_REPEAT;
-        hfit &= op.rx() <= (op.mode == KF_MIRROR101 ? kStreamV - 1 : kStreamV);
+        hfit &= op.rx() <= (op.mode == KF_MIRROR101 ? kV_ - 1 : kV_);
     }
     si.edge_v = !rep && p->H >= 4 * si.L + 2 * si.P + 8;
     // unrolled: ~P copies per variant (4 variants + 2 peeled prologues); too
@@ -2048,9 +2072,9 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     // the rolled loop), unless KFUSE_ROLLED_EDGE_V=0 leaves those rows to the
     // frame: for deep10 the frame's index-exchange tiles cost 12 % of the kernel
     if (si.rolled && !env_int("KFUSE_ROLLED_EDGE_V", 1, 0, 1)) si.edge_v = false;
-    si.edge_l = !rep && hfit && p->W >= 4 * kStreamV;
+    si.edge_l = !rep && hfit && p->W >= 4 * kV_;
     si.edge_r = si.edge_l && si.vec;
-    si.ok = b.Rx <= 2 * kStreamV * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
+    si.ok = b.Rx <= 2 * kV_ * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
     return si;
 }
 

@@ -137,7 +137,8 @@ struct Separable {                // rank-1 mask: m[j][i] = col[j] * row[i]
 // Interior streaming schedule of one block (codegen.cpp StreamGen)
 struct StreamInfo {
     bool ok = false;              // the block has an interior fast path
-    bool vec = false;             // W % 4 == 0: 128-bit loads/stores
+    int V = 4;                    // pixels per lane of the interior path (4, or 8 for f32 with KFUSE_V8)
+    bool vec = false;             // W % V == 0: 128-bit loads/stores
     int L = 0;                    // rows of lag of the sink behind the newest input row
     int HL = 1;                   // halo lanes per warp side
     int P = 1;                    // ring period = loop body copies

@@ -256,7 +256,7 @@ void prepare(kf_pipeline *p, kf_plan *plan)
 // whole waves of resident warps.  Returns the grid size.
 static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlock &cb)
 {
-    const int W = a.W, H = a.H, V = kStreamV;
+    const int W = a.W, H = a.H, V = cb.si.V;
     const StreamInfo &si = cb.si;
     int fx0 = 0, fx1 = 0, fy0 = 0, fy1 = 0;
     bool fast = si.ok, top = false, bot = false;
