@@ -403,3 +403,38 @@ def test_strip_geometry_bit_identical(wl, monkeypatch):
     for ns in (2, 5, 40, 118):
         monkeypatch.setenv("KFUSE_NSTRIPS", str(ns))
         np.testing.assert_array_equal(run_gpu(spec, plan, ins)[0], base)
+
+
+# Code-generation / launch knobs that change how the same arithmetic is
+# scheduled: results must stay bit-identical to the default.
+SAME_BITS = ["KFUSE_V8=1", "KFUSE_PERSIST=1", "KFUSE_QPTR=0", "KFUSE_LDS_PF=0", "KFUSE_CONST_W=0",
+             "KFUSE_HEAVY_FIRST=0", "KFUSE_PRO_RP=0", "KFUSE_SMEM_ROWS=6"]
+
+
+@pytest.mark.parametrize("wl", ["harris", "deep10", "unsharp"])
+@pytest.mark.parametrize("knob", SAME_BITS)
+def test_schedule_knobs_bit_identical(wl, knob, monkeypatch):
+    spec = P.WORKLOADS[wl](200, 150)
+    ins = _inputs(spec, 12)
+    base = run_gpu(spec, make_plan(spec, "b200"), ins)[0]
+    k, v = knob.split("=")
+    monkeypatch.setenv(k, v)
+    got = run_gpu(spec, make_plan(spec, "b200"), ins)[0]
+    np.testing.assert_array_equal(got, base)
+
+
+@pytest.mark.parametrize("wl", ["deep10", "harris"])
+def test_rolled_edges_left_to_frame_still_exact(wl, monkeypatch):
+    """KFUSE_ROLLED_EDGE_V=0 and a tiny code budget (rolled body) move rows between
+    the streaming path and the frame tiles: u8x4 stays bit-exact, f32 within TOL."""
+    spec = P.WORKLOADS[wl](130, 97)
+    ins = _inputs(spec, 13)
+    ref = O.run(spec, ins)[spec["outputs"][0]]
+    for env in ({"KFUSE_ROLLED_EDGE_V": "0"}, {"KFUSE_CODE_BUDGET": "1000"},
+                {"KFUSE_CODE_BUDGET": "1000", "KFUSE_ROLLED_EDGE_V": "0"}):
+        for k, v in env.items():
+            monkeypatch.setenv(k, v)
+        got = run_gpu(spec, make_plan(spec, "b200"), ins)[0]
+        check(spec, got, ref, f"{wl} {env}")
+        for k in env:
+            monkeypatch.delenv(k)
