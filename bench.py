@@ -467,6 +467,36 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
         dist.all_reduce(agree, op=dist.ReduceOp.MIN)
         if int(agree.item()) == 0 and mode == "peer":
             mode, halo, note = "nccl", None, "peer setup failed on another rank; "
+    if mode == "peer" and (halo.up is not None or halo.down is not None):
+        # Self-check on this hardware before timing: the buffers were generated
+        # with their halo rows, so kf_run_band over them is the reference.  Poison
+        # the halo rows, run one peer step, and require the same bits; else every
+        # rank falls back to NCCL (and says so in the JSON line).
+        ok = 1
+        try:
+            ref_out = torch.empty_like(outs[0])
+            plan.run_band(band.row0, band.row1, [ins[0]], band.in0, band.in1, [ref_out], stream)
+            torch.cuda.synchronize()
+            t_, n_ = band.top, band.rows
+            if gspec["dtype"] == "f32":
+                ins[0][:t_].fill_(float("nan"))
+                ins[0][t_ + n_:].fill_(float("nan"))
+            else:
+                ins[0][:t_].fill_(77)
+                ins[0][t_ + n_:].fill_(77)
+            chk = torch.empty_like(outs[0])
+            dist.barrier()
+            halo.step(plan, 0, [chk], stream, side)
+            torch.cuda.synchronize()
+            ok = int(halo.errors() == 0 and torch.equal(chk, ref_out))
+        except Exception as e:   # noqa: BLE001 -- any failure means: do not use the peer path
+            note += f"peer self-check raised {type(e).__name__}; "
+            ok = 0
+        agree = torch.tensor([ok], dtype=torch.int32, device="cuda" if dist.get_backend() == "nccl" else "cpu")
+        dist.all_reduce(agree, op=dist.ReduceOp.MIN)
+        if int(agree.item()) == 0:
+            mode, halo, note = "nccl", None, note + "peer self-check failed; "
+            ins[0].copy_(torch.from_numpy(host).to(ins[0].device))   # restore the halo rows
     (c0, c1), edges = KD.split_rows(band)
     exch = halo is not None and (halo.up is not None or halo.down is not None)
     launches_per_step = plan.num_launches * ((1 if c1 > c0 else 0) + len(edges)) + (2 if exch else 0)
