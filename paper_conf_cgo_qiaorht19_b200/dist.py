@@ -229,29 +229,38 @@ class PeerHalo:
         K.peer_wait(cnt, [self._c(_SENT)] * len(cnt), self._c(_ERR), self.spin, stream)
 
     def step(self, plan, s: int, outputs, stream, side=None) -> None:
-        """One band step on buffer set s: core rows on `stream` while `side`
-        (a second stream, forked from `stream`) signals and pulls the halo rows;
-        then the edge strips on `stream`.  Bit-identical to exchange_halos +
-        run_band.  With side=None everything runs on `stream`, in the order
-        signal, core, pull, edges.  Without neighbours it is just the core."""
+        """One band step on buffer set s: the core rows on `stream` while `side`
+        (a second stream, forked from `stream`) signals, pulls the halo rows and
+        computes the edge strips -- they read only the pulled and the own rows and
+        write rows disjoint from the core's, so the whole exchange hides behind
+        the core; `stream` joins `side` at the end.  Bit-identical to
+        exchange_halos + run_band.  With side=None everything runs on `stream`,
+        in the order signal, core, pull, edges.  Without neighbours it is just
+        the core."""
         b = self.band
         (c0, c1), edges = split_rows(b)
         ins = [self.bufs[s]]
         exch = self.up is not None or self.down is not None
+
+        def run_edges(st):
+            for r0, r1 in edges:
+                plan.run_band(r0, r1, ins, b.in0, b.in1, [o[r0 - b.row0:r1 - b.row0] for o in outputs], st)
+
         if exch and side is not None:
             side.wait_stream(stream)          # the own rows of this step are ready
             self.signal(side)
             self.pull(s, side)
+            run_edges(side)
         elif exch:
             self.signal(stream)
         if c1 > c0:
             plan.run_band(c0, c1, ins, b.in0, b.in1, [o[c0 - b.row0:c1 - b.row0] for o in outputs], stream)
         if exch and side is not None:
             stream.wait_stream(side)
-        elif exch:
-            self.pull(s, stream)
-        for r0, r1 in edges:
-            plan.run_band(r0, r1, ins, b.in0, b.in1, [o[r0 - b.row0:r1 - b.row0] for o in outputs], stream)
+        else:
+            if exch:
+                self.pull(s, stream)
+            run_edges(stream)
 
     def close(self) -> None:
         """Drops the peer mappings.  Call on every rank (synchronised) before any
