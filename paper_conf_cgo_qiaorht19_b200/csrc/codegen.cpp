@@ -1676,8 +1676,13 @@ struct StreamGen {
         // strip bounds in primed (streaming-direction) rows
         // balanced strips: strip i covers rows [fy0 + i*Hf/ns, fy0 + (i+1)*Hf/ns)
         o << "    const int Hf = a.fy1 - a.fy0;\n";
-        o << "    const int ys0 = a.fy0 + (int)((long long)strip * Hf / a.n_strips);\n";
-        o << "    const int ye0 = a.fy0 + (int)((long long)(strip + 1) * Hf / a.n_strips);\n";
+        // two strip heights (tail split): strip s starts at unit u(s) = 2s for s <= n_long,
+        // s + n_long after; Hf is spread over n_strips + n_long units (n_long = 0: balanced)
+        o << "    const int nu = a.n_strips + a.n_long;\n";
+        o << "    const int u0 = strip <= a.n_long ? 2 * strip : strip + a.n_long;\n";
+        o << "    const int u1 = strip + 1 <= a.n_long ? 2 * strip + 2 : strip + 1 + a.n_long;\n";
+        o << "    const int ys0 = a.fy0 + (int)((long long)u0 * Hf / nu);\n";
+        o << "    const int ye0 = a.fy0 + (int)((long long)u1 * Hf / nu);\n";
         if (dir > 0) {
             o << "    const int ys = ys0, ye = ye0;\n";
         } else {

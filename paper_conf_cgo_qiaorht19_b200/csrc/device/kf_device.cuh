@@ -39,6 +39,7 @@ struct KfArgs {
     int n_strips;                  // row strips (the last one takes the remainder)
     int n_items;                   // n_chunks * n_strips
     int edge_l, edge_r, edge_t, edge_b;   // image edges handled by the edge chunks / strips
+    int n_long;                    // strips [0, n_long) are two units tall, the rest one unit
 };
 
 // ------------------------------------------------------------ border map

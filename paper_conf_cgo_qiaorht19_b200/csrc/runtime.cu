@@ -319,6 +319,14 @@ static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlo
         best_ns = std::max(min_strips, std::min(force, std::max(min_strips, Hf / smin)));
     a.n_strips = best_ns;
     a.strip = (Hf + best_ns - 1) / best_ns;
+    // Optional tail split (KFUSE_NLONG = n): the first n strips are two units
+    // tall and the rest one unit, so the last wave runs short items.  Edge
+    // strips must still hold smin rows.  Off by default.
+    a.n_long = 0;
+    if (const int nl = env_int("KFUSE_NLONG", 0, 0, 1 << 20)) {
+        int n = std::min(nl, best_ns - 1);
+        if (n > 0 && Hf / (best_ns + n) >= smin) a.n_long = n;
+    }
     a.n_items = a.n_chunks * a.n_strips;
     return (unsigned)(cta + a.n_items);
 }
