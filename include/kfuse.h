@@ -22,7 +22,9 @@
  *     human-readable, thread-local message in kf_last_error().
  *   - Image ids are dense int32 in declaration order: inputs first, then each
  *     kernel's output image (kernel k writes image n_inputs + k).
- *   - Images are dense, row-major, pitch = width * 4 bytes, 16-byte aligned:
+ *   - Images are dense, row-major, pitch = width * 4 bytes.  Base pointers
+ *     must be 16-byte aligned when width % 4 == 0 (128-bit row access), else
+ *     4-byte aligned (any row offset of a larger image works):
  *       KF_F32  : one float32 per pixel (gray)
  *       KF_U8X4 : one uchar4 per pixel (interleaved RGBA; each channel is an
  *                 independent image with identical kernels, int32 arithmetic)
@@ -31,7 +33,11 @@
  *     and compiled modules.
  *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
  *   - Not thread-safe per pipeline; distinct pipelines may be used from
- *     distinct threads.
+ *     distinct threads.  A plan with more than one block keeps its cut-edge
+ *     intermediates in ONE workspace: two kf_run / kf_run_band calls of such a
+ *     plan must not be in flight on different streams at the same time
+ *     (single-block plans write only their outputs and may overlap on
+ *     disjoint output rows).
  */
 #ifndef KFUSE_H
 #define KFUSE_H
@@ -157,6 +163,23 @@ kf_status kf_add_local_op(kf_pipeline *p, int32_t input, const double *mask, int
 /* Pipeline outputs are external outputs for legality (Fig. 2c). */
 kf_status kf_mark_output(kf_pipeline *p, int32_t image_id);
 
+/* ---- schedule options -------------------------------------------------------
+ * Per-pipeline integer options that change how the fused kernels are
+ * SCHEDULED (code shape, input feed, launch geometry), never what they
+ * compute: for every option the output is bit-identical to the default (GPU
+ * test test_schedule_options_bit_identical).  No environment variable reaches
+ * the library; this is the only tuning interface (DESIGN.md §5.4 lists the
+ * options and their measurements).  Code-generation options take effect for
+ * plans prepared afterwards; run-time options (nstrips, host_taper) at the next
+ * kf_run.  Names: swar swring swring_cap pairs defer prefetch sring smem_rows
+ * lds_pf const_w pro_rp qptr heavy_first code_budget rolled_edge_v minctas
+ * nstrips host_taper.  Unknown names or out-of-range values: KF_ERR_ARG.
+ * (The measured-and-rejected v8 / persist / persist_waves / nlong exist only
+ * in a KF_EXPERIMENTAL build, and the naive_border negative control only in
+ * the KF_TEST_HOOKS build libkfuse_testhooks.so, never in libkfuse.so.) */
+kf_status kf_set_option(kf_pipeline *p, const char *name, int64_t value);
+kf_status kf_get_option(const kf_pipeline *p, const char *name, int64_t *value);
+
 /* ---- planning (host only; freezes the graph) ---------------------------- */
 /* Alg. 1 GetLegalPartitions with the benefit model. */
 kf_status kf_plan_fusion(kf_pipeline *p, const kf_model_params *m, kf_plan **out);
@@ -265,11 +288,14 @@ kf_status kf_run_band(kf_pipeline *p, const kf_plan *plan, int32_t row0, int32_t
  * it on `stream`; increments *sent (local, nullable). */
 kf_status kf_peer_signal(uint32_t *const *flags, int32_t n, uint32_t *sent, void *stream);
 
-/* For each segment i: wait until *flag[i] passes *seen[i], copy bytes[i] bytes
- * from src[i] (the neighbour's boundary rows) to dst[i] (the local halo rows),
- * set *seen[i] += 1, then release-increment ack[i] (the neighbour's "consumed"
- * counter; ack may be null). */
-kf_status kf_peer_pull(int32_t n, void *const *dst, const void *const *src, const int64_t *bytes,
+/* For each segment i < n (one per neighbour): wait until *flag[i] passes
+ * *seen[i], then for each copy c < m (one per pipeline input image) copy
+ * bytes[i*m+c] bytes from src[i*m+c] (the neighbour's boundary rows) to
+ * dst[i*m+c] (the local halo rows), set *seen[i] += 1, then release-increment
+ * ack[i] (the neighbour's "consumed" counter; ack may be null).  Any
+ * alignment is accepted (16-B vectors when both ends are 16-B aligned, else
+ * 4-B words or bytes).  n <= 4, 1 <= m <= 8. */
+kf_status kf_peer_pull(int32_t n, int32_t m, void *const *dst, const void *const *src, const int64_t *bytes,
                        uint32_t *const *flag, uint32_t *const *seen, uint32_t *const *ack, uint32_t *err,
                        int64_t spin_limit, void *stream);
 

@@ -234,6 +234,18 @@ def swar_stress(W, H, mode="mirror"):
     return p.spec()
 
 
+def two_input(width: int, height: int, mode: str = "clamp") -> dict:
+    """Test workload with two input images (multi-input row bands / peer halos):
+    a 5x5 binomial blur of input 0, a Sobel-x of input 1, combined pointwise with
+    input 0 (a shared external input, Fig. 2b shape)."""
+    p = Pipeline("two_input", width, height, "f32")
+    a, b = p.input(), p.input()
+    bl = p.local("blur", a, [[v / 256.0 for v in r] for r in outer(BINOM5, BINOM5)], mode)
+    dx = p.local("dx", b, SOBEL_X, mode)
+    p.output(p.point("mix", [bl, dx, a], [L(0), L(1), MUL, L(2), ADD]))
+    return p.spec()
+
+
 def fig4(mode: str = "clamp") -> dict:
     """Fig. 4: two unnormalised 3x3 Gaussian local kernels on a 5x5 image."""
     p = Pipeline("fig4", 5, 5, "f32")
@@ -252,9 +264,13 @@ MODES = ["clamp", "mirror", "mirror101", "repeat", "constant"]
 
 
 def random_pipeline(rng: random.Random, width: int, height: int, dtype: str, n_kernels: int,
-                    modes=None, max_radius: int = 2) -> dict:
+                    modes=None, max_radius: int = 2, asym: float = 0.0) -> dict:
     """Random connected DAG of point/local kernels for property tests.  Values stay
-    bounded: f32 programs are convex-ish combinations, u8x4 programs saturate."""
+    bounded: f32 programs are convex-ish combinations, u8x4 programs saturate.
+    max_radius bounds each mask's radius per axis; with probability `asym` a local
+    kernel takes a strongly asymmetric shape instead (1x7, 9x1, 1x9, 7x1, 3x7, 9x5
+    masks as (rows x cols)).  asym = 0 draws no extra random numbers, so the
+    default stream of DAGs is unchanged."""
     modes = modes or MODES
     p = Pipeline(f"rand_{dtype}_{n_kernels}", width, height, dtype)
     n_in = rng.choice([1, 1, 2])
@@ -270,6 +286,8 @@ def random_pipeline(rng: random.Random, width: int, height: int, dtype: str, n_k
             rx = rng.choice([r, rng.randint(0, max_radius)])
             if rx == 0 and ry == 0:
                 rx = 1
+            if asym and rng.random() < asym:
+                ry, rx = rng.choice([(0, 3), (4, 0), (0, 4), (3, 0), (1, 3), (4, 2)])
             mode = rng.choice(modes)
             src = pick()
             if dtype == "f32":
@@ -338,6 +356,7 @@ WORKLOADS = {
     "deep10": deep10,
     "copy": copy,
     "blur": blur,
+    "two_input": two_input,
 }
 
 # BASELINE.json configs: (workload, W, H, seed)

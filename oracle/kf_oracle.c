@@ -30,12 +30,20 @@
  * int32, the GPU's accumulator width) and every kernel output is saturated to
  * [0,255] when it is stored (narrowing at every kernel boundary).
  *
- * Built with -O2 -ffp-contract=off.
+ * Built with -O2 -ffp-contract=off -fopenmp.  Threads: or_set_threads(n) (1 =
+ * the plain serial loop).  With n > 1 the ROWS of one kernel are split over
+ * threads (each pixel is still computed by exactly the code below, in the same
+ * order of taps); kernels still run one after another.  This is the SURVEY
+ * §8(d) "OpenMP over rows on all cores" baseline mode and makes full-size
+ * element-by-element parity affordable; it changes no arithmetic.
  */
 #include <math.h>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 /* ---- op-IR opcodes (restated from include/kfuse.h kf_opcode) ---------- */
 enum {
@@ -65,6 +73,21 @@ typedef struct {
 } or_op;
 
 static int g_err;            /* sticky: 1 = int32 overflow, 2 = bad program */
+static int g_threads = 1;
+
+static void set_err(int e) { __atomic_store_n(&g_err, e, __ATOMIC_RELAXED); }
+
+/* Number of threads for or_run / or_eval_points (<= 0: all cores). Returns it. */
+int or_set_threads(int n)
+{
+#ifdef _OPENMP
+    g_threads = n > 0 ? n : omp_get_num_procs();
+#else
+    g_threads = 1;
+    (void)n;
+#endif
+    return g_threads;
+}
 
 /* ---- border map, -1 = constant ---------------------- */
 int or_border(int p, int n, int mode)
@@ -117,16 +140,17 @@ static double run_f(const or_op *o, int n, const int *op, const int *arg, const 
             st[sp++] = a < b ? b : (a > c ? c : a); break;
         case OR_SELECT_GT: { double d = st[--sp]; c = st[--sp]; b = st[--sp]; a = st[--sp];
             st[sp++] = a > b ? c : d; break; }
-        default: g_err = 2; return 0.0;   /* SHR/SHL/SAT/LUT are integer-only */
+        default: set_err(2); return 0.0;   /* SHR/SHL/SAT/LUT are integer-only */
         }
     }
     (void)o;
-    return sp == 1 ? st[0] : (g_err = 2, 0.0);
+    if (sp != 1) set_err(2);
+    return sp == 1 ? st[0] : 0.0;
 }
 
 static int64_t chk(int64_t v)
 {
-    if (v > INT32_MAX || v < INT32_MIN) g_err = 1;
+    if (v > INT32_MAX || v < INT32_MIN) set_err(1);
     return v;
 }
 
@@ -165,10 +189,11 @@ static int64_t run_i(const or_op *o, int n, const int *op, const int *arg, const
             if (a < 0) a = 0;
             if (a >= o->lut_len) a = o->lut_len - 1;
             st[sp++] = o->lut[a]; break;
-        default: g_err = 2; return 0;
+        default: set_err(2); return 0;
         }
     }
-    return sp == 1 ? st[0] : (g_err = 2, 0);
+    if (sp != 1) set_err(2);
+    return sp == 1 ? st[0] : 0;
 }
 
 static int64_t sat_u8(int64_t v) { return v < 0 ? 0 : (v > 255 ? 255 : v); }
@@ -194,9 +219,10 @@ static int64_t pload_i(void *vc, int k)
 static void exec_op(int W, int H, int dtype, void **img, const or_op *o, void *out)
 {
     int nc = dtype == OR_F32 ? 1 : 4;
-    pctx ctx;
-    ctx.img = img; ctx.W = W; ctx.o = o;
-    for (int y = 0; y < H; y++)
+#pragma omp parallel for schedule(static) num_threads(g_threads) if (g_threads > 1)
+    for (int y = 0; y < H; y++) {
+        pctx ctx;
+        ctx.img = img; ctx.W = W; ctx.o = o;
         for (int x = 0; x < W; x++)
             for (int c = 0; c < nc; c++) {
                 ctx.x = x; ctx.y = y; ctx.c = c;
@@ -236,6 +262,7 @@ static void exec_op(int W, int H, int dtype, void **img, const or_op *o, void *o
                             sat_u8(run_i(o, o->n_prog, o->prog_op, o->prog_arg, o->prog_imm, pload_i, &ctx));
                 }
             }
+    }
 }
 
 /*
@@ -359,6 +386,7 @@ int or_eval_points(int W, int H, int dtype, int n_inputs, const void *const *inp
     ectx e = {W, H, dtype, n_inputs, inputs, ops};
     (void)n_ops;
     g_err = 0;
+#pragma omp parallel for schedule(dynamic, 16) num_threads(g_threads) if (g_threads > 1)
     for (int i = 0; i < n; i++) {
         if (dtype == OR_F32) ((double *)out)[i] = ev_f(&e, id, ys[i], xs[i]);
         else for (int c = 0; c < 4; c++) ((uint8_t *)out)[i * 4 + c] = (uint8_t)ev_i(&e, id, ys[i], xs[i], c);

@@ -9,6 +9,7 @@ eval_points(spec, inputs, id, ys, xs) -> recursive pointwise evaluation (same
                                    definition; index-exchange semantics,
                                    PAPER.md:1088-1133)
 border(p, n, mode)              -> the border index map
+set_threads(n)                  -> OpenMP threads over rows (1 = serial)
 """
 from __future__ import annotations
 
@@ -46,8 +47,8 @@ def build(force: bool = False) -> str:
     with _lock:
         if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
             tmp = _LIB + f".{os.getpid()}.tmp"
-            subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fPIC", "-shared", "-std=c11",
-                                   "-o", tmp, _SRC, "-lm"])
+            subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared",
+                                   "-std=c11", "-o", tmp, _SRC, "-lm"])
             os.replace(tmp, _LIB)
     return _LIB
 
@@ -60,8 +61,19 @@ def _load():
         lib.or_eval_points.restype = C.c_int
         lib.or_border.restype = C.c_int
         lib.or_border.argtypes = [C.c_int, C.c_int, C.c_int]
+        lib.or_set_threads.restype = C.c_int
+        lib.or_set_threads.argtypes = [C.c_int]
+        # default: all cores (rows of each kernel split over threads; no arithmetic change),
+        # or $KF_ORACLE_THREADS
+        lib.or_set_threads(int(os.environ.get("KF_ORACLE_THREADS", "0")))
         _lib = lib
     return _lib
+
+
+def set_threads(n: int) -> int:
+    """Threads used by run()/eval_points(): 1 = the serial loop, <= 0 = all cores.
+    Returns the number actually used."""
+    return int(_load().or_set_threads(int(n)))
 
 
 def border(p: int, n: int, mode: str) -> int:

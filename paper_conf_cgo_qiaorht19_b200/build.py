@@ -45,37 +45,65 @@ def _digest(paths) -> str:
     return h.hexdigest()
 
 
+# The product library, and a test-only variant with the negative-control hook
+# (option naive_border: pad-once fusion, Fig. 4b) and the measured-and-rejected
+# experimental options.  Only tests load the variant.
+VARIANTS = {
+    "libkfuse.so": [],
+    "libkfuse_testhooks.so": ["-DKF_TEST_HOOKS", "-DKF_EXPERIMENTAL"],
+}
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
-    os.makedirs(BUILD, exist_ok=True)
+    from concurrent.futures import ThreadPoolExecutor
     _embed_header()
+    with ThreadPoolExecutor(len(VARIANTS)) as ex:   # the variants build in parallel (nvcc is serial per file)
+        for f in [ex.submit(_build_variant, os.path.join(PKG, name), defs, force, verbose)
+                  for name, defs in VARIANTS.items()]:
+            f.result()
+    return os.path.join(PKG, "libkfuse.so")
+
+
+def _build_variant(lib_path: str, defs: list, force: bool, verbose: bool) -> str:
+    bdir = BUILD if not defs else BUILD + "_" + os.path.basename(lib_path).split(".")[0]
+    os.makedirs(bdir, exist_ok=True)
     headers = [os.path.join(CSRC, "kf_internal.h"), os.path.join(CSRC, "kf_device_cuh.inc"),
                os.path.join(ROOT, "include", "kfuse.h")]
-    objs = []
+    objs, jobs = [], []
     for s in SOURCES:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(BUILD, s + ".o")
+        obj = os.path.join(bdir, s + ".o")
         stamp = obj + ".sha"
-        dig = _digest([src] + headers)
+        dig = _digest([src] + headers) + " ".join(defs)
         objs.append(obj)
         if not force and os.path.exists(obj) and os.path.exists(stamp) and open(stamp).read() == dig:
             continue
-        cmd = [NVCC] + ARCH + FLAGS + ["-c", src, "-o", obj]
+        cmd = [NVCC] + ARCH + FLAGS + defs + ["-c", src, "-o", obj]
         if s.endswith(".cpp"):
-            cmd = [NVCC] + ARCH + FLAGS + ["-x", "cu", "-c", src, "-o", obj]
+            cmd = [NVCC] + ARCH + FLAGS + defs + ["-x", "cu", "-c", src, "-o", obj]
+        jobs.append((cmd, stamp, dig))
+
+    def compile_one(job):
+        cmd, stamp, dig = job
         if verbose:
             print(" ".join(cmd))
         subprocess.check_call(cmd)
         with open(stamp, "w") as f:
             f.write(dig)
-    tmp = LIB + f".{os.getpid()}.tmp"
+
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max(1, min(len(jobs), os.cpu_count() or 1))) as ex:
+        for f in [ex.submit(compile_one, j) for j in jobs]:
+            f.result()
+    tmp = lib_path + f".{os.getpid()}.tmp"
     cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + [
         "-L/usr/local/cuda/lib64", "-lnvrtc", "-lcudart_static", "-ldl", "-lrt", "-lpthread",
         "-Xlinker", "-rpath=/usr/local/cuda/lib64"]
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib_path)
+    return lib_path
 
 
 if __name__ == "__main__":

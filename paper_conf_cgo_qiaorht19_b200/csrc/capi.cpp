@@ -363,6 +363,29 @@ kf_status kf_run_band(kf_pipeline *p, const kf_plan *plan, int32_t row0, int32_t
 }
 
 const char *kf_last_error(void) { return g_last_error.c_str(); }
-const char *kf_version(void) { return "kfuse 0.1 (sm_100a)"; }
+kf_status kf_set_option(kf_pipeline *p, const char *name, int64_t value)
+{
+    return guard([&] {
+        if (!p) fail(KF_ERR_ARG, "null pipeline");
+        set_option(p, name, (long long)value);
+    });
+}
+
+kf_status kf_get_option(const kf_pipeline *p, const char *name, int64_t *value)
+{
+    return guard([&] {
+        if (!p || !value) fail(KF_ERR_ARG, "null pipeline or value");
+        *value = (int64_t)get_option(p, name);
+    });
+}
+
+const char *kf_version(void)
+{
+#ifdef KF_TEST_HOOKS
+    return "kfuse 0.2 (sm_100a) TEST HOOKS BUILD -- negative controls, not the product library";
+#else
+    return "kfuse 0.2 (sm_100a)";
+#endif
+}
 
 }  // extern "C"

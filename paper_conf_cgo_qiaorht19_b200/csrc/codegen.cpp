@@ -29,6 +29,7 @@
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 #include <functional>
 #include <numeric>
 #include <sstream>
@@ -680,9 +681,21 @@ struct FrameGen {
     int tmp = 0;
     int TW = 32, TH = 8;
     ProgEmitter pe;
+    bool naive = false;      // negative control only (option naive_border, KF_TEST_HOOKS build)
+    int naive_mode = KF_CLAMP;
+    double naive_const = 0.0;
 
     FrameGen(const kf_pipeline *p_, const BlockInfo &b_, int block_, std::ostringstream &o_)
-        : p(p_), b(b_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp} {}
+        : p(p_), b(b_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp}
+    {
+        naive = !b.torus && opt(p, "naive_border");
+        for (int k : b.kernels)
+            if (p->ops[k].kind == LOCAL) {   // "pad once": the input is padded with the first local kernel's mode
+                naive_mode = p->ops[k].mode;
+                naive_const = p->ops[k].constant;
+                break;
+            }
+    }
 
     std::string KV() const { return f32 ? "float" : "I4"; }
     std::string var() { return "v" + std::to_string(tmp++); }
@@ -716,6 +729,17 @@ struct FrameGen {
         if (!in_block(img)) {
             std::string Y = "y", X = "x";
             if (b.torus) { Y = "kf_wrap(y, H)"; X = "kf_wrap(x, W)"; }
+            if (naive) {   // negative control: the padded input plane at (y, x)
+                const std::string md = std::to_string(naive_mode);
+                std::string yy = var(), xx = var();
+                o << ind << "const int " << yy << " = kf_border<" << md << ">(y, H);\n";
+                o << ind << "const int " << xx << " = kf_border<" << md << ">(x, W);\n";
+                std::string c = f32 ? fconst(naive_const) : "kf_i4(" + iconst((int)naive_const) + ")";
+                o << ind << "const " << KV() << " " << v << " = (" << yy << " < 0 || " << xx << " < 0) ? " << c
+                  << " : " << ext_load(img, yy, xx) << ";\n";
+                memo[img] = v;
+                return v;
+            }
             o << ind << "const " << KV() << " " << v << " = " << ext_load(img, Y, X) << ";\n";
             memo[img] = v;
             return v;
@@ -744,7 +768,7 @@ struct FrameGen {
                     const int dy = j - cy, dx = i - cx;
                     std::string Y = "y + (" + std::to_string(dy) + ")", X = "x + (" + std::to_string(dx) + ")";
                     std::string val;
-                    if (b.torus && staged_in) {
+                    if ((b.torus || naive) && staged_in) {   // naive: no index exchange (Fig. 4b)
                         val = smem_load(in - p->n_inputs, Y, X);
                     } else if (b.torus) {
                         val = ext_load(in, "kf_wrap(" + Y + ", H)", "kf_wrap(" + X + ", W)");
@@ -798,7 +822,9 @@ struct FrameGen {
             o << "    for (int i = threadIdx.x; i < " << rw * rh << "; i += blockDim.x) {\n";
             o << "        const int y = oy - " << hy << " + i / " << rw << ", x = ox - " << hx << " + i % " << rw
               << ";\n";
-            if (!b.torus)
+            if (naive)
+                o << "        if (y < a.r0 - " << hy << " || y >= a.r1 + " << hy << ") continue;\n";
+            else if (!b.torus)
                 o << "        if (y < 0 || y >= H || x < 0 || x >= W || y < a.r0 - " << hy << " || y >= a.r1 + "
                   << hy << ") continue;\n";
             std::map<int, std::string> memo;
@@ -928,7 +954,7 @@ struct StreamGen {
     bool pm = false;   // f32 values kept as packed pixel pairs (F2) for column-local math
     bool runptr = false;   // steady-state loop uses running row pointers (set per variant)
     bool vedge = false;    // variant starts at an image edge (peeled iterations remap taps)
-    bool defer_ok = true;  // pair mode: defer normalised masks' power-of-two scales (KFUSE_DEFER)
+    bool defer_ok = true;  // pair mode: defer normalised masks' power-of-two scales (option "defer")
     std::set<int> prp;     // external images fed by running row pointers from the prologue on (interior strips)
     bool qptr = false;     // steady-state loop: ring slots addressed from per-trip base pointers
 
@@ -1667,7 +1693,7 @@ struct StreamGen {
         o << "    const int lane = threadIdx.x & 31;\n";
         // The image size is fixed per pipeline (one iteration space):
         // baked in, row strides become immediates and unrolled rows use address offsets.
-        if (env_int("KFUSE_CONST_W", 1, 0, 1))
+        if (opt(p, "const_w"))
             o << "    constexpr int W = " << p->W << ", H = " << p->H << ";\n    (void)H;\n";
         else
             o << "    const int W = a.W, H = a.H;\n    (void)H;\n";
@@ -1717,7 +1743,7 @@ struct StreamGen {
         // launch geometry keeps inside [base, rlast]: no clamps, one running
         // pointer from the first prologue row on.
         prp.clear();
-        if (si.sring && !ve && dir > 0 && env_int("KFUSE_PRO_RP", 1, 0, 1))
+        if (si.sring && !ve && dir > 0 && opt(p, "pro_rp"))
             for (int img : b.ext)
                 if (HY(img) == L) prp.insert(img);
         if (!prp.empty()) {
@@ -1796,7 +1822,7 @@ struct StreamGen {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
             if (si.lpf) o << "        const int qnext = qb + " << P << " == " << si.DS << " ? 0 : qb + " << P << ";\n";
-            qptr = si.sring && env_int("KFUSE_QPTR", 1, 0, 1);
+            qptr = si.sring && opt(p, "qptr");
             if (qptr)
                 for (int img : b.ext) {
                     const int s = slot.at(img);
@@ -1816,8 +1842,8 @@ struct StreamGen {
     void run()
     {
         for (size_t i = 0; i < b.ext.size(); i++) slot[b.ext[i]] = (int)i;
-        pm = f32 && env_int("KFUSE_PAIRS", 1, 0, 1);
-        defer_ok = env_int("KFUSE_DEFER", 1, 0, 1);
+        pm = f32 && opt(p, "pairs");
+        defer_ok = opt(p, "defer");
 
         // Variants (the variant is CTA-uniform):
         //   interior strip, interior chunk   -- the hot loop, no border logic
@@ -1832,7 +1858,7 @@ struct StreamGen {
             variant(-1, true, si.edge_l, si.edge_r);
         }
         o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast(const KfArgs &a, const int item)\n{\n";
-        if (env_int("KFUSE_HEAVY_FIRST", 1, 0, 1)) {
+        if (opt(p, "heavy_first")) {
             // heavy items first: the edge strips (longer peeled prologues) and the
             // edge chunks (lane selects) start in the first wave instead of
             // forming the tail of the last one
@@ -1927,13 +1953,91 @@ static Separable factor(const Op &op, bool integer)
     return s;
 }
 
-// Tuning knobs (diagnostics / sweeps): integer env var in [lo, hi] or the default.
-int env_int(const char *name, int dflt, int lo, int hi)
+// Schedule options.  They change how the same arithmetic is
+// scheduled -- code shape, feed, launch geometry -- never its result: every
+// option is covered by a GPU test that checks the output is bit-identical to
+// the default.  Set per pipeline through kf_set_option (no environment
+// variable reaches the library).  The measured-and-rejected alternatives
+// (v8, persist, persist_waves, nlong) exist only in the KF_EXPERIMENTAL build.
+namespace {
+struct OptDef { const char *name; long long dflt, lo, hi; bool experimental; };
+const OptDef kOpts[] = {
+    {"swar", 1, 0, 1, false},           // u8x4 kernels in SWAR form (§5.2b)
+    {"swring", 1, 0, 1, false},         // unpacked SWAR rings
+    {"swring_cap", 164, 0, 1024, false},
+    {"pairs", 1, 0, 1, false},          // f32 packed pixel pairs (FFMA2/FADD2)
+    {"defer", 1, 0, 1, false},          // deferred power-of-two mask scales
+    {"prefetch", 4, 1, 16, false},      // register prefetch distance (no smem ring)
+    {"sring", 1, 0, 1, false},          // cp.async shared-memory row ring
+    {"smem_rows", 12, 2, 64, false},    // rows of that ring
+    {"lds_pf", 1, 0, 1, false},         // ring rows read one iteration ahead
+    {"const_w", 1, 0, 1, false},        // image size baked into the kernel
+    {"pro_rp", 1, 0, 1, false},         // running row pointer from the prologue on
+    {"qptr", 1, 0, 1, false},           // per-trip ring slot base pointers
+    {"heavy_first", 1, 0, 1, false},    // edge items first
+    {"code_budget", 12000, 0, 1 << 30, false},   // unrolled vs rolled body
+    {"rolled_edge_v", 1, 0, 1, false},  // rolled bodies keep the edge strips
+    {"minctas", kMinCtasPerSm, 1, 32, false},    // __launch_bounds__ min CTAs per SM
+    {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)
+    {"host_taper", 1, 0, 1, false},     // kf_run_host thin first/last bands
+    {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
+    {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
+    {"persist_waves", 1, 1, 1 << 20, true},
+    {"nlong", 0, 0, 1 << 20, true},     // tail split (rejected)
+    // NEGATIVE CONTROL ONLY: settable in libkfuse_testhooks.so (KF_TEST_HOOKS),
+    // never in the product library, where it is always 0.  The frame path then
+    // evaluates in-block producers on the padded plane instead of remapping each
+    // consumer tap -- the "pad once" fusion of Fig. 4b, which is WRONG at the
+    // border.  Tests assert it fails parity.
+    {"naive_border", 0, 0, 1, true},
+};
+#ifdef KF_EXPERIMENTAL
+constexpr bool kExperimental = true;
+#else
+constexpr bool kExperimental = false;
+#endif
+#ifdef KF_TEST_HOOKS
+constexpr bool kTestHooks = true;
+#else
+constexpr bool kTestHooks = false;
+#endif
+const OptDef *find_opt(const char *name)   // settable options of this build
 {
-    const char *e = std::getenv(name);
-    if (!e || !*e) return dflt;
-    int v = std::atoi(e);
-    return std::min(hi, std::max(lo, v));
+    for (const OptDef &d : kOpts)
+        if (!std::strcmp(d.name, name)) {
+            if (!std::strcmp(name, "naive_border")) return kTestHooks ? &d : nullptr;
+            return (d.experimental && !kExperimental) ? nullptr : &d;
+        }
+    return nullptr;
+}
+}  // namespace
+
+long long opt(const kf_pipeline *p, const char *name)
+{
+    const OptDef *d = find_opt(name);
+    if (!d) {
+        for (const OptDef &e : kOpts)
+            if (!std::strcmp(e.name, name)) return e.dflt;   // experimental option, not built in
+        fail(KF_ERR_ARG, std::string("internal: unknown option ") + name);
+    }
+    auto it = p->options.find(name);
+    return it == p->options.end() ? d->dflt : it->second;
+}
+
+void set_option(kf_pipeline *p, const char *name, long long value)
+{
+    const OptDef *d = name ? find_opt(name) : nullptr;
+    if (!d) fail(KF_ERR_ARG, std::string("unknown option '") + (name ? name : "(null)") + "'");
+    if (value < d->lo || value > d->hi)
+        fail(KF_ERR_ARG, std::string("option '") + name + "' out of range [" + std::to_string(d->lo) + ", " +
+                             std::to_string(d->hi) + "]");
+    p->options[name] = value;
+}
+
+long long get_option(const kf_pipeline *p, const char *name)
+{
+    if (!name || !find_opt(name)) fail(KF_ERR_ARG, std::string("unknown option '") + (name ? name : "(null)") + "'");
+    return opt(p, name);
 }
 
 // Code-size weight of a program: SASS instructions its opcodes expand to
@@ -1960,7 +2064,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     StreamInfo si;
     // f32 blocks may run 8 pixels per lane (two float4 per row per lane):
     // half the shuffles and per-row overhead per pixel, twice the ring registers
-    si.V = (p->dtype == KF_F32 && env_int("KFUSE_V8", 0, 0, 1)) ? 8 : kStreamV;
+    si.V = (p->dtype == KF_F32 && opt(p, "v8")) ? 8 : kStreamV;
     const int kV_ = si.V;
     si.vec = p->W % kV_ == 0;
     for (int img : b.ext) si.hy[img] = b.ext_hy.at(img);
@@ -1978,7 +2082,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
             si.depth[in] = std::max(si.depth[in], d);
         }
         if (op.kind == LOCAL) si.sep[k] = factor(op, p->dtype != KF_F32);
-        if (p->dtype == KF_U8X4 && env_int("KFUSE_SWAR", 1, 0, 1) &&
+        if (p->dtype == KF_U8X4 && opt(p, "swar") &&
             swar_feasible(op, op.kind == LOCAL ? si.sep[k] : Separable{}))
             si.swk.insert(k);
     }
@@ -1989,11 +2093,11 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     // input feed: a cp.async shared-memory ring of DS rows per external image
     // (128-bit rows), else register prefetch D iterations ahead.  Ring period
     // P >= every depth (+ D for register-prefetched external images).
-    si.D = env_int("KFUSE_PREFETCH", 4, 1, 16);
-    si.sring = si.vec && env_int("KFUSE_SRING", 1, 0, 1) && !b.ext.empty();
+    si.D = (int)opt(p, "prefetch");
+    si.sring = si.vec && opt(p, "sring") && !b.ext.empty();
     if (si.sring) {
         si.P = std::max(maxdepth, maxdepth_ext);
-        const int want = env_int("KFUSE_SMEM_ROWS", 12, 2, 64);
+        const int want = (int)opt(p, "smem_rows");
         const int cap = 32768 / (128 * kV_ * (int)b.ext.size());   // <= 32 KB of ring per warp
         int DS = std::max(want, si.P + 1);
         DS = (DS + si.P - 1) / si.P * si.P;
@@ -2001,7 +2105,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         if (DS > cap || DS < 2) si.sring = false;
         si.DS = DS;
         si.ring_bytes = (int)b.ext.size() * DS * 128 * kV_;
-        si.lpf = si.sring && DS >= 3 && env_int("KFUSE_LDS_PF", 1, 0, 1);
+        si.lpf = si.sring && DS >= 3 && opt(p, "lds_pf");
     }
     if (!si.sring) si.P = std::max(maxdepth, maxdepth_ext + si.D);
     // register estimate: live ring values (depth per image, D prefetched rows)
@@ -2016,8 +2120,8 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     // pixel) at every row use.  Costs depth x V more registers; deepest first,
     // under a cap on the live ring registers.
     const int live_packed = live;
-    if (p->dtype == KF_U8X4 && env_int("KFUSE_SWRING", 1, 0, 1)) {
-        const int cap = env_int("KFUSE_SWRING_CAP", 164, 0, 1024);
+    if (p->dtype == KF_U8X4 && opt(p, "swring")) {
+        const int cap = (int)opt(p, "swring_cap");
         std::vector<std::pair<int, int>> cand;   // (depth, image)
         for (auto &kv : si.depth) {
             const int img = kv.first;
@@ -2071,15 +2175,16 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     // unrolled: ~P copies per variant (4 variants + 2 peeled prologues); too
     // much straight-line code for NVRTC/ptxas and the instruction cache ->
     // one rolled body copy
-    const long long budget = env_int("KFUSE_CODE_BUDGET", 12000, 0, 1 << 30);
+    const long long budget = opt(p, "code_budget");
     si.rolled = ops * si.P * 6 > budget;
     // rolled bodies keep the edge strips too (peeled remapped prologue, then
-    // the rolled loop), unless KFUSE_ROLLED_EDGE_V=0 leaves those rows to the
+    // the rolled loop), unless option rolled_edge_v=0 leaves those rows to the
     // frame: for deep10 the frame's index-exchange tiles cost 12 % of the kernel
-    if (si.rolled && !env_int("KFUSE_ROLLED_EDGE_V", 1, 0, 1)) si.edge_v = false;
+    if (si.rolled && !opt(p, "rolled_edge_v")) si.edge_v = false;
     si.edge_l = !rep && hfit && p->W >= 4 * kV_;
     si.edge_r = si.edge_l && si.vec;
     si.ok = b.Rx <= 2 * kV_ * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
+    if (opt(p, "naive_border")) si.ok = false;   // negative control: everything through the (naive) frame
     return si;
 }
 
@@ -2117,7 +2222,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
         StreamGen sg(p, b, si, block, o);
         sg.run();
     }
-    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << env_int("KFUSE_MINCTAS", kMinCtasPerSm, 1, 32) << ") " << kernel_name(b, block)
+    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << opt(p, "minctas") << ") " << kernel_name(b, block)
       << "(const __grid_constant__ KfArgs a)\n{\n";
     // Persistent CTAs: the grid is at most one wave of resident CTAs, and each
     // loops over work items (frame tiles first, then interior items) with a

@@ -52,6 +52,7 @@ struct kf_pipeline {
     std::vector<int> outputs;     // marked output image ids, in marking order
     bool frozen = false;
     kf::Runtime *rt = nullptr;    // owned; created lazily by the runtime
+    std::map<std::string, long long> options;   // kf_set_option (schedule options, codegen.cpp)
     ~kf_pipeline();
     int n_images() const { return n_inputs + (int)ops.size(); }
     bool is_kernel_image(int id) const { return id >= n_inputs; }
@@ -137,7 +138,7 @@ struct Separable {                // rank-1 mask: m[j][i] = col[j] * row[i]
 // Interior streaming schedule of one block (codegen.cpp StreamGen)
 struct StreamInfo {
     bool ok = false;              // the block has an interior fast path
-    int V = 4;                    // pixels per lane of the interior path (4, or 8 for f32 with KFUSE_V8)
+    int V = 4;                    // pixels per lane of the interior path (4, or 8 for f32 with option v8)
     bool vec = false;             // W % V == 0: 128-bit loads/stores
     int L = 0;                    // rows of lag of the sink behind the newest input row
     int HL = 1;                   // halo lanes per warp side
@@ -160,14 +161,16 @@ struct StreamInfo {
 };
 
 std::string kernel_name(const BlockInfo &b, int block);
-int env_int(const char *name, int dflt, int lo, int hi);
+long long opt(const kf_pipeline *p, const char *name);          // option value or its default
+void set_option(kf_pipeline *p, const char *name, long long value);
+long long get_option(const kf_pipeline *p, const char *name);
 StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b);
 std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block);
 
 // runtime.cu
 void prepare(kf_pipeline *p, kf_plan *plan);
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
-         void *stream, int row0, int row1, int in_row0, int in_row1);
+         void *stream, int row0, int row1, int in_row0, int in_row1, bool out_full = false);
 void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
               void *stream);
 void release_plan(kf_plan *plan);

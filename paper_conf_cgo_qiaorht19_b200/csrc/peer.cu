@@ -33,10 +33,13 @@ struct SigArgs {
     unsigned *sent;            // local count of signals (nullable)
     int n;
 };
+constexpr int kMaxCopy = 8;   // copies per segment (one per pipeline input)
+
 struct PullArgs {
-    void *dst[kMaxSeg];
-    const void *src[kMaxSeg];  // peer rows
-    long long bytes[kMaxSeg];
+    void *dst[kMaxSeg][kMaxCopy];
+    const void *src[kMaxSeg][kMaxCopy];   // peer rows
+    long long bytes[kMaxSeg][kMaxCopy];
+    int m;                     // copies per segment
     unsigned *flag[kMaxSeg];   // local counter written by the neighbour
     unsigned *seen[kMaxSeg];   // local count of pulls done
     unsigned *ack[kMaxSeg];    // neighbour's ack counter (peer, nullable)
@@ -94,13 +97,30 @@ __global__ void __launch_bounds__(512) peer_pull_k(const __grid_constant__ PullA
     }
     __syncthreads();   // the acquire of thread 0 orders the copies below (causality via bar.sync)
     if (!ok) return;
-    const long long n16 = a.bytes[s] >> 4;
-    const int4 *src = (const int4 *)a.src[s];
-    int4 *dst = (int4 *)a.dst[s];
-    for (long long i = threadIdx.x; i < n16; i += blockDim.x) dst[i] = __ldcv(src + i);   // NVLink P2P loads
-    const char *sb = (const char *)a.src[s];
-    char *db = (char *)a.dst[s];
-    for (long long i = (n16 << 4) + threadIdx.x; i < a.bytes[s]; i += blockDim.x) db[i] = sb[i];
+    for (int c = 0; c < a.m; c++) {
+        // 16-B vectors when both ends are 16-B aligned (rows of a W % 4 == 0
+        // image), else 4-B words (any f32 / uchar4 row offset), else bytes;
+        // then the tail.
+        const uintptr_t al = (uintptr_t)a.src[s][c] | (uintptr_t)a.dst[s][c];
+        const char *sb = (const char *)a.src[s][c];
+        char *db = (char *)a.dst[s][c];
+        const long long nb = a.bytes[s][c];
+        long long done = 0;
+        if ((al & 15) == 0) {
+            const long long n16 = nb >> 4;
+            const int4 *src = (const int4 *)sb;
+            int4 *dst = (int4 *)db;
+            for (long long i = threadIdx.x; i < n16; i += blockDim.x) dst[i] = __ldcv(src + i);   // NVLink P2P loads
+            done = n16 << 4;
+        } else if ((al & 3) == 0) {
+            const long long n4 = nb >> 2;
+            const unsigned *src = (const unsigned *)sb;
+            unsigned *dst = (unsigned *)db;
+            for (long long i = threadIdx.x; i < n4; i += blockDim.x) dst[i] = __ldcv(src + i);
+            done = n4 << 2;
+        }
+        for (long long i = done + threadIdx.x; i < nb; i += blockDim.x) db[i] = sb[i];
+    }
     __syncthreads();
     if (threadIdx.x == 0) {
         *a.seen[s] = want;
@@ -143,24 +163,32 @@ extern "C" kf_status kf_peer_signal(uint32_t *const *flags, int32_t n, uint32_t 
     KF_GUARD(peer_signal_k<<<1, 32, 0, (cudaStream_t)stream>>>(a));
 }
 
-extern "C" kf_status kf_peer_pull(int32_t n, void *const *dst, const void *const *src, const int64_t *bytes,
-                                  uint32_t *const *flag, uint32_t *const *seen, uint32_t *const *ack, uint32_t *err,
-                                  int64_t spin_limit, void *stream)
+extern "C" kf_status kf_peer_pull(int32_t n, int32_t m, void *const *dst, const void *const *src,
+                                  const int64_t *bytes, uint32_t *const *flag, uint32_t *const *seen,
+                                  uint32_t *const *ack, uint32_t *err, int64_t spin_limit, void *stream)
 {
-    if (n < 0 || n > kMaxSeg || !err || (n && (!dst || !src || !bytes || !flag || !seen))) {
-        set_error("kf_peer_pull: bad arguments");
+    if (n < 0 || n > kMaxSeg || m < 1 || m > kMaxCopy || !err || (n && (!dst || !src || !bytes || !flag || !seen))) {
+        set_error("kf_peer_pull: bad arguments (0..4 segments of 1..8 copies)");
         return KF_ERR_ARG;
     }
     if (n == 0) return KF_OK;
     PullArgs a{};
+    a.m = m;
     for (int i = 0; i < n; i++) {
-        if (!dst[i] || !src[i] || bytes[i] < 0 || !flag[i] || !seen[i]) {
-            set_error("kf_peer_pull: null segment");
+        if (!flag[i] || !seen[i]) {
+            set_error("kf_peer_pull: null counter");
             return KF_ERR_ARG;
         }
-        a.dst[i] = dst[i];
-        a.src[i] = src[i];
-        a.bytes[i] = bytes[i];
+        for (int c = 0; c < m; c++) {
+            const int j = i * m + c;
+            if (!dst[j] || !src[j] || bytes[j] < 0) {
+                set_error("kf_peer_pull: null copy");
+                return KF_ERR_ARG;
+            }
+            a.dst[i][c] = dst[j];
+            a.src[i][c] = src[j];
+            a.bytes[i][c] = bytes[j];
+        }
         a.flag[i] = flag[i];
         a.seen[i] = seen[i];
         a.ack[i] = ack ? ack[i] : nullptr;

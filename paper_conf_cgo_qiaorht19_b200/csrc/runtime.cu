@@ -254,7 +254,7 @@ void prepare(kf_pipeline *p, kf_plan *plan)
 // tiled by the shared-memory index-exchange path.  One warp (= one CTA) per
 // (column chunk, row strip) item; the strip height is chosen so the items fill
 // whole waves of resident warps.  Returns the grid size.
-static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlock &cb)
+static unsigned launch_geometry(const kf_pipeline *p, KfArgs &a, const BlockInfo &b, const CompiledBlock &cb)
 {
     const int W = a.W, H = a.H, V = cb.si.V;
     const StreamInfo &si = cb.si;
@@ -315,15 +315,16 @@ static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlo
         if (best < 0 || cost < best - 1e-9) { best = cost; best_ns = ns; }
         if (items > 64 * slots) break;
     }
-    if (const int force = env_int("KFUSE_NSTRIPS", 0, 0, 1 << 20))   // tuning / diagnostics
+    if (const int force = (int)opt(p, "nstrips"))   // schedule option (sweeps; results unchanged)
         best_ns = std::max(min_strips, std::min(force, std::max(min_strips, Hf / smin)));
     a.n_strips = best_ns;
     a.strip = (Hf + best_ns - 1) / best_ns;
-    // Optional tail split (KFUSE_NLONG = n): the first n strips are two units
-    // tall and the rest one unit, so the last wave runs short items.  Edge
-    // strips must still hold smin rows.  Off by default.
+    // Optional tail split (experimental option "nlong" = n): the first n strips
+    // are two units tall and the rest one unit, so the last wave runs short
+    // items.  Edge strips must still hold smin rows.  Measured slower, so only in
+    // the KF_EXPERIMENTAL build.
     a.n_long = 0;
-    if (const int nl = env_int("KFUSE_NLONG", 0, 0, 1 << 20)) {
+    if (const int nl = (int)opt(p, "nlong")) {
         int n = std::min(nl, best_ns - 1);
         if (n > 0 && Hf / (best_ns + n) >= smin) a.n_long = n;
     }
@@ -332,14 +333,23 @@ static unsigned launch_geometry(KfArgs &a, const BlockInfo &b, const CompiledBlo
 }
 
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
-         void *stream, int row0, int row1, int in_row0, int in_row1)
+         void *stream, int row0, int row1, int in_row0, int in_row1, bool out_full)
 {
     if (n_in != p->n_inputs || (n_in && !din)) fail(KF_ERR_ARG, "wrong number of inputs");
     if (n_out != (int)p->outputs.size() || (n_out && !dout)) fail(KF_ERR_ARG, "wrong number of outputs");
+    // 128-bit row access (the interior path's vector loads/stores) needs 16-B
+    // aligned rows, i.e. 16-B aligned base pointers when W % 4 == 0; otherwise
+    // the kernels access single 4-B pixels and any 4-B aligned pointer works
+    // (e.g. a row offset into a larger image).
+    const uintptr_t amask = p->W % 4 == 0 ? 15 : 3;
     for (int i = 0; i < n_in; i++)
-        if (!din[i] || ((uintptr_t)din[i] & 15)) fail(KF_ERR_ARG, "input pointers must be non-null, 16-B aligned");
+        if (!din[i] || ((uintptr_t)din[i] & amask))
+            fail(KF_ERR_ARG, amask == 15 ? "input pointers must be non-null, 16-B aligned"
+                                         : "input pointers must be non-null, 4-B aligned");
     for (int j = 0; j < n_out; j++)
-        if (!dout[j] || ((uintptr_t)dout[j] & 15)) fail(KF_ERR_ARG, "output pointers must be non-null, 16-B aligned");
+        if (!dout[j] || ((uintptr_t)dout[j] & amask))
+            fail(KF_ERR_ARG, amask == 15 ? "output pointers must be non-null, 16-B aligned"
+                                         : "output pointers must be non-null, 4-B aligned");
     prepare(p, plan);
     Driver &d = driver();
     const bool band = !(row0 == 0 && row1 == p->H && in_row0 == 0);
@@ -375,7 +385,7 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
             band_copies.push_back({o, j});
         } else {
             ptr[o] = dout[j];
-            base[o] = band ? row0 : 0;
+            base[o] = band && !out_full ? row0 : 0;   // out_full: dout holds the whole image
         }
     }
     CUstream st = (CUstream)stream;
@@ -398,19 +408,15 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         a.r0 = blo[bi];
         a.r1 = bhi[bi];
         if (a.r1 <= a.r0) continue;
-        unsigned grid = launch_geometry(a, b, cb);
+        unsigned grid = launch_geometry(p, a, b, cb);
         if (!cb.si.ok) a.n_items = 0;   // frame-only block
-        if (const char *skip = getenv("KFUSE_DIAG_SKIP")) {   // timing diagnostics only: wrong results
-            if (!strcmp(skip, "frame")) { grid -= a.frame_ctas; a.frame_ctas = 0; a.n_rect = 0; }
-            if (!strcmp(skip, "fast")) { grid = a.frame_ctas; a.n_items = 0; }
-        }
-        {   // Optional persistent CTAs (KFUSE_PERSIST=1): at most one wave, the kernel
-            // strides over the items.  Off by default: measured slower (C3 27.4 ->
+        {   // Optional persistent CTAs (experimental option "persist"): at most one
+            // wave, the kernel strides over the items.  Measured slower (C3 27.4 ->
             // 30.0 us, C4 327 -> 363; profiles/r01_sweep_persist.jsonl) -- the
-            // hardware refilling freed CTA slots balances better than a static stride.
-            const long long slots = (long long)cb.num_sms * cb.ctas_per_sm *
-                                    env_int("KFUSE_PERSIST_WAVES", 1, 1, 1 << 20);
-            if (env_int("KFUSE_PERSIST", 0, 0, 1) && (long long)grid > slots) grid = (unsigned)slots;
+            // hardware refilling freed CTA slots balances better than a static
+            // stride -- so only in the KF_EXPERIMENTAL build.
+            const long long slots = (long long)cb.num_sms * cb.ctas_per_sm * opt(p, "persist_waves");
+            if (opt(p, "persist") && (long long)grid > slots) grid = (unsigned)slots;
         }
         if (grid == 0) continue;
         void *params[] = {&a};
@@ -418,7 +424,8 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
     }
     for (auto &c : band_copies) {
         const char *src = (const char *)plan->workspace[c.first] + (size_t)row0 * p->W * 4;
-        KF_CUDA(cudaMemcpyAsync(dout[c.second], src, (size_t)(row1 - row0) * p->W * 4, cudaMemcpyDeviceToDevice,
+        char *dst = (char *)dout[c.second] + (out_full ? (size_t)row0 * p->W * 4 : 0);
+        KF_CUDA(cudaMemcpyAsync(dst, src, (size_t)(row1 - row0) * p->W * 4, cudaMemcpyDeviceToDevice,
                                 (cudaStream_t)stream));
     }
 }
@@ -474,7 +481,7 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     // ends are thin: row shares 1,3,6,6,6,6,3,1 / 32 (uniform when fewer bands).
     static const int kShare8[9] = {0, 1, 4, 10, 16, 22, 28, 31, 32};
     auto cut = [&](int k) {
-        if (nb == kHostBands && kHostBands == 8 && env_int("KFUSE_HOST_TAPER", 1, 0, 1))
+        if (nb == kHostBands && kHostBands == 8 && opt(p, "host_taper"))
             return (int)((long long)p->H * kShare8[k] / 32);
         return (int)((long long)p->H * k / nb);
     };
@@ -490,12 +497,13 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
         }
         KF_CUDA(cudaEventRecord(rt.ev_in[k], rt.s_h2d));
         KF_CUDA(cudaStreamWaitEvent(s, rt.ev_in[k], 0));
-        std::vector<void *> dout(n_out);
-        for (int j = 0; j < n_out; j++) dout[j] = nb == 1 ? rt.stage_out[j] : (char *)rt.stage_out[j] + r0 * row_bytes;
+        // the band writes rows [r0, r1) of the whole staging image (out_full): a
+        // pointer offset to row r0 would not be 16-B aligned when W % 4 != 0
+        std::vector<void *> dout(rt.stage_out.begin(), rt.stage_out.end());
         if (nb == 1)
             run(p, plan, din.data(), n_in, dout.data(), n_out, stream, 0, p->H, 0, p->H);
         else
-            run(p, plan, din.data(), n_in, dout.data(), n_out, stream, r0, r1, 0, p->H);
+            run(p, plan, din.data(), n_in, dout.data(), n_out, stream, r0, r1, 0, p->H, true);
         KF_CUDA(cudaEventRecord(rt.ev_out[k], s));
         KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_out[k], 0));
         for (int j = 0; j < n_out; j++)

@@ -93,6 +93,10 @@ def run_step_overlapped(plan, band: Band, inputs, outputs, side_stream, group=No
     edges in every call)."""
     cur = torch.cuda.current_stream()
     (c0, c1), edges = split_rows(band)
+    if plan.num_launches > 1:
+        # a multi-block plan keeps its intermediates in one workspace: the core
+        # and edge calls must not overlap (kfuse.h), so the core runs on `cur`
+        side_stream = cur
     side_stream.wait_stream(cur)                      # inputs of this step are ready
     reqs = []
     if band.world > 1 and band.halo > 0:
@@ -146,19 +150,24 @@ class PeerHalo:
     (torch.multiprocessing's CUDA IPC reductions, exchanged once with
     all_gather_object) and runs the band steps over them.
 
-    bufs: this rank's rotating input buffers, each holding rows [in0, in1) of
-    the global image (first dim = rows).  Every rank must pass the same number
-    of buffers, and call step() the same number of times with the same set
-    indices, in the same order."""
+    bufs: this rank's rotating input buffer SETS.  A set is one tensor (a
+    one-input pipeline) or a list with one tensor per pipeline input; each
+    tensor holds rows [in0, in1) of its global image (first dim = rows).  Every
+    rank must pass the same number of sets of the same shape, and call step()
+    the same number of times with the same set indices, in the same order."""
 
     def __init__(self, band: Band, bufs, group=None, spin_limit: int = 1 << 27):
         from torch.multiprocessing.reductions import reduce_tensor
-        self.band, self.bufs, self.spin = band, list(bufs), spin_limit
-        self.ctr = torch.zeros(8, dtype=torch.int32, device=self.bufs[0].device)
+        self.band, self.spin = band, spin_limit
+        self.bufs = [list(s) if isinstance(s, (list, tuple)) else [s] for s in bufs]
+        if len({len(s) for s in self.bufs}) != 1 or not 1 <= len(self.bufs[0]) <= 8:
+            raise ValueError("every buffer set must hold the same number (1..8) of input tensors")
+        dev = self.bufs[0][0].device
+        self.ctr = torch.zeros(8, dtype=torch.int32, device=dev)
         if band.world == 1:   # no neighbours: nothing to share
             self.up = self.down = None
             return
-        mine = {"ctr": reduce_tensor(self.ctr), "bufs": [reduce_tensor(b) for b in self.bufs],
+        mine = {"ctr": reduce_tensor(self.ctr), "bufs": [[reduce_tensor(t) for t in s] for s in self.bufs],
                 "top": band.top, "rows": band.rows}
         every = [None] * band.world
         dist.all_gather_object(every, mine, group=group)
@@ -169,14 +178,15 @@ class PeerHalo:
 
         def peer(r):
             d = every[r]
-            return {"ctr": open_(d["ctr"]), "bufs": [open_(x) for x in d["bufs"]], "top": d["top"], "rows": d["rows"]}
+            return {"ctr": open_(d["ctr"]), "bufs": [[open_(x) for x in s] for s in d["bufs"]], "top": d["top"],
+                    "rows": d["rows"]}
 
         self.up = peer(band.rank - 1) if band.rank > 0 and band.top > 0 else None
         self.down = peer(band.rank + 1) if band.rank < band.world - 1 and band.bottom > 0 else None
         # the pull/signal kernels run on this rank's GPU and touch the
         # neighbours' memory directly: enable the P2P path (NVLink) explicitly
         from . import kfuse as K
-        dev = self.bufs[0].device.index
+        dev = dev.index
         for nb in (self.up, self.down):
             if nb is not None:
                 K.peer_enable(dev, nb["ctr"].device.index)
@@ -201,26 +211,29 @@ class PeerHalo:
     def pull(self, s: int, stream) -> None:
         """Copies the neighbours' boundary rows of buffer set s into the halo rows."""
         from . import kfuse as K
-        b, buf = self.band, self.bufs[s]
-        rb = buf[0].numel() * buf.element_size()
+        b, bset = self.band, self.bufs[s]
         dst, src, nb, flag, seen, ack = [], [], [], [], [], []
-        if self.up:
+        if self.up:   # one segment per neighbour, one copy per input image
             u = self.up
-            dst.append(buf.data_ptr())
-            src.append(u["bufs"][s].data_ptr() + (u["top"] + u["rows"] - b.top) * rb)
-            nb.append(b.top * rb)
+            for i, buf in enumerate(bset):
+                rb = buf[0].numel() * buf.element_size()
+                dst.append(buf.data_ptr())
+                src.append(u["bufs"][s][i].data_ptr() + (u["top"] + u["rows"] - b.top) * rb)
+                nb.append(b.top * rb)
             flag.append(self._c(_READY_ABOVE))
             seen.append(self._c(_SEEN_ABOVE))
             ack.append(self._c(_ACK_BELOW, u["ctr"]))
         if self.down:
             d = self.down
-            dst.append(buf.data_ptr() + (b.top + b.rows) * rb)
-            src.append(d["bufs"][s].data_ptr() + d["top"] * rb)
-            nb.append(b.bottom * rb)
+            for i, buf in enumerate(bset):
+                rb = buf[0].numel() * buf.element_size()
+                dst.append(buf.data_ptr() + (b.top + b.rows) * rb)
+                src.append(d["bufs"][s][i].data_ptr() + d["top"] * rb)
+                nb.append(b.bottom * rb)
             flag.append(self._c(_READY_BELOW))
             seen.append(self._c(_SEEN_BELOW))
             ack.append(self._c(_ACK_ABOVE, d["ctr"]))
-        K.peer_pull(dst, src, nb, flag, seen, ack, self._c(_ERR), self.spin, stream)
+        K.peer_pull(dst, src, nb, flag, seen, ack, self._c(_ERR), self.spin, stream, copies=len(bset))
 
     def wait_consumed(self, stream) -> None:
         """Before the own rows are overwritten: both neighbours pulled every step signalled."""
@@ -239,8 +252,10 @@ class PeerHalo:
         the core."""
         b = self.band
         (c0, c1), edges = split_rows(b)
-        ins = [self.bufs[s]]
+        ins = self.bufs[s]
         exch = self.up is not None or self.down is not None
+        if plan.num_launches > 1:
+            side = None   # one workspace per plan: core and edges must not overlap (kfuse.h)
 
         def run_edges(st):
             for r0, r1 in edges:

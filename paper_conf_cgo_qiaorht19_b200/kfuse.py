@@ -17,7 +17,6 @@ if not os.path.exists(_LIBPATH):
     raise ImportError(f"libkfuse.so not built at {_LIBPATH}: run "
                       "`python -m paper_conf_cgo_qiaorht19_b200.build` (or __graft_entry__.build())")
 
-lib = C.CDLL(_LIBPATH)
 
 KF_F32, KF_U8X4 = 0, 1
 DTYPES = {"f32": KF_F32, "u8x4": KF_U8X4}
@@ -66,7 +65,7 @@ _SIGS = {
     "kf_plan_fusion": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
     "kf_plan_basic": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
     "kf_peer_signal": (C.c_int, [_P, C.c_int32, _P, _P]),
-    "kf_peer_pull": (C.c_int, [C.c_int32, _P, _P, _P, _P, _P, _P, _P, C.c_int64, _P]),
+    "kf_peer_pull": (C.c_int, [C.c_int32, C.c_int32, _P, _P, _P, _P, _P, _P, _P, C.c_int64, _P]),
     "kf_peer_wait": (C.c_int, [C.c_int32, _P, _P, _P, C.c_int64, _P]),
     "kf_peer_enable": (C.c_int, [C.c_int32, C.c_int32]),
     "kf_plan_exact": (C.c_int, [_P, C.POINTER(ModelParams), C.POINTER(_P)]),
@@ -88,13 +87,24 @@ _SIGS = {
     "kf_run_host": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_band": (C.c_int, [_P, _P, C.c_int32, C.c_int32, C.POINTER(_P), C.c_int32, C.c_int32,
                               C.POINTER(_P), _P]),
+    "kf_set_option": (C.c_int, [_P, C.c_char_p, C.c_int64]),
+    "kf_get_option": (C.c_int, [_P, C.c_char_p, C.POINTER(C.c_int64)]),
     "kf_last_error": (C.c_char_p, []),
     "kf_version": (C.c_char_p, []),
 }
-for _n, (_r, _a) in _SIGS.items():
-    _f = getattr(lib, _n)
-    _f.restype = _r
-    _f.argtypes = _a
+
+
+def _open(path: str) -> C.CDLL:
+    """Loads a libkfuse build and declares the C-ABI signatures."""
+    lb = C.CDLL(path)
+    for n, (r, a) in _SIGS.items():
+        f = getattr(lb, n)
+        f.restype = r
+        f.argtypes = a
+    return lb
+
+
+lib = _open(_LIBPATH)
 
 EXPORTED = sorted(_SIGS)
 
@@ -181,10 +191,22 @@ class Pipeline:
         _check(lib.kf_mark_output(self.h, int(img)))
         self.outputs.append(int(img))
 
+    def set_option(self, name: str, value: int) -> None:
+        """kf_set_option: a schedule option (results are bit-identical for every value)."""
+        _check(lib.kf_set_option(self.h, name.encode(), int(value)))
+
+    def get_option(self, name: str) -> int:
+        v = C.c_int64()
+        _check(lib.kf_get_option(self.h, name.encode(), C.byref(v)))
+        return v.value
+
     @classmethod
-    def from_spec(cls, spec: dict) -> "Pipeline":
-        """Builds the pipeline of a plain-data description (kf_inputs.pipelines)."""
+    def from_spec(cls, spec: dict, options: dict | None = None) -> "Pipeline":
+        """Builds the pipeline of a plain-data description (kf_inputs.pipelines),
+        with optional schedule options {name: value}."""
         p = cls(spec["width"], spec["height"], spec["dtype"])
+        for name, value in (options or {}).items():
+            p.set_option(name, value)
         for _ in range(spec["n_inputs"]):
             p.add_input()
         for o in spec["ops"]:
@@ -329,10 +351,12 @@ def peer_signal(flags, sent=0, stream=None) -> None:
     _check(lib.kf_peer_signal(_ptrs(flags), len(flags), _P(int(sent)), _P(_stream(stream))))
 
 
-def peer_pull(dst, src, nbytes, flag, seen, ack, err, spin_limit=1 << 27, stream=None) -> None:
-    """kf_peer_pull over len(dst) segments (all arguments device addresses; ack entries may be 0)."""
-    _check(lib.kf_peer_pull(len(dst), _ptrs(dst), _ptrs(src), _i64s(nbytes), _ptrs(flag), _ptrs(seen),
-                            _ptrs(ack), _P(int(err)), int(spin_limit), _P(_stream(stream))))
+def peer_pull(dst, src, nbytes, flag, seen, ack, err, spin_limit=1 << 27, stream=None, copies=1) -> None:
+    """kf_peer_pull over len(flag) segments of `copies` copies each (dst/src/nbytes
+    hold len(flag) * copies entries, segment-major; all arguments device
+    addresses; ack entries may be 0)."""
+    _check(lib.kf_peer_pull(len(flag), int(copies), _ptrs(dst), _ptrs(src), _i64s(nbytes), _ptrs(flag),
+                            _ptrs(seen), _ptrs(ack), _P(int(err)), int(spin_limit), _P(_stream(stream))))
 
 
 def peer_wait(counter, target, err, spin_limit=1 << 27, stream=None) -> None:

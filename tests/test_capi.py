@@ -231,7 +231,7 @@ def test_exact_planner_size_limit():
 def test_swar_form_chosen_by_interval_analysis():
     """u8x4 codegen: kernels whose lanes provably fit 16 bits run
     two channels per op (PRMT-unpacked SWAR); a 16-bit-overflowing mask, ABS, DIV,
-    SELECT and a variable product fall back to per-channel int32; KFUSE_SWAR=0
+    SELECT and a variable product fall back to per-channel int32; option swar=0
     turns the form off."""
     spec = P.swar_stress(64, 48)
     plan = K.Pipeline.from_spec(spec).plan_unfused()
@@ -241,12 +241,38 @@ def test_swar_form_chosen_by_interval_analysis():
         form[spec["ops"][b]["name"]] = "swar" if "__byte_perm" in body else "int32"
     assert form == {"a": "swar", "b": "swar", "c": "swar", "d": "swar", "e": "int32", "f": "int32",
                     "g": "int32", "h": "int32", "k": "int32", "m": "swar"}
-    os.environ["KFUSE_SWAR"] = "0"
-    try:
-        plan = K.Pipeline.from_spec(spec).plan_unfused()
-        assert all("__byte_perm" not in plan.source(b).split("_fast_di(")[1] for b in range(plan.num_launches))
-    finally:
-        del os.environ["KFUSE_SWAR"]
+    plan = K.Pipeline.from_spec(spec, {"swar": 0}).plan_unfused()
+    assert all("__byte_perm" not in plan.source(b).split("_fast_di(")[1] for b in range(plan.num_launches))
     c4, _ = P.config("C4")
     src = K.Pipeline.from_spec(c4).plan_fusion("b200").source(0).split("_fast_di(")[1]
     assert "kf_unpack" not in src and "kf_lut(" not in src   # all ten deep10 kernels in SWAR form
+
+
+def test_schedule_options_api():
+    """kf_set_option / kf_get_option: known options with defaults and ranges; unknown
+    names, out-of-range values and the test-only / experimental options are
+    rejected by the product library (no environment variable reaches it)."""
+    p = K.Pipeline(64, 32)
+    assert p.get_option("smem_rows") == 12 and p.get_option("swar") == 1
+    p.set_option("smem_rows", 6)
+    assert p.get_option("smem_rows") == 6
+    for bad in ("naive_border", "v8", "persist", "nlong", "no_such_option", "KFUSE_SWAR"):
+        with pytest.raises(K.KfError) as e:
+            p.set_option(bad, 1)
+        assert e.value.name == "KF_ERR_ARG"
+    with pytest.raises(K.KfError):
+        p.set_option("smem_rows", 1000)
+    assert "TEST HOOKS" not in K.version()
+
+
+def test_library_reads_no_environment():
+    """The product library's only getenv is the cubin cache directory: no knob can
+    change what kf_run computes."""
+    import subprocess
+    so = os.path.join(os.path.dirname(K.__file__), "libkfuse.so")
+    syms = subprocess.run(["nm", "-D", "--undefined-only", so], capture_output=True, text=True).stdout
+    strings = subprocess.run(["strings", so], capture_output=True, text=True).stdout.split()
+    assert "KFUSE_CACHE_DIR" in strings
+    assert not [t for t in strings if t.startswith("KFUSE_") and t != "KFUSE_CACHE_DIR"], \
+        [t for t in strings if t.startswith("KFUSE_")]
+    assert "getenv" in syms

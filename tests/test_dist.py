@@ -48,34 +48,40 @@ def test_partition_rejects_band_thinner_than_halo():
         KD.partition(8, 4, 1, 3)
 
 
-def _worker(rank, world, port, H, W, halo, q, posted=False):
+def _worker(rank, world, port, H, W, halo, q, posted=False, n_inputs=1):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         band = KD.partition(H, world, rank, halo)
-        full = gen.image_f32(9, W, H)
-        buf = torch.full((band.in1 - band.in0, W), float("nan"))
-        own = torch.from_numpy(full[band.row0:band.row1])
-        buf[band.top:band.top + band.rows] = own
-        if posted:   # the overlapped step's non-blocking post (dist.run_step_overlapped)
-            for r in KD._post_halos([buf], band):
+        fulls = [gen.image_f32(9 + 13 * j, W, H) for j in range(n_inputs)]
+        bufs = []
+        for full in fulls:
+            buf = torch.full((band.in1 - band.in0, W), float("nan"))
+            buf[band.top:band.top + band.rows] = torch.from_numpy(full[band.row0:band.row1])
+            bufs.append(buf)
+        if posted:   # the overlapped step's non-blocking post (dist.run_step_overlapped), all inputs at once
+            for r in KD._post_halos(bufs, band):
                 r.wait()
         else:
-            KD.exchange_halos(buf, band)
-        ok = bool(np.array_equal(buf.numpy(), full[band.in0:band.in1]))
+            for buf in bufs:
+                KD.exchange_halos(buf, band)
+        ok = all(bool(np.array_equal(b.numpy(), f[band.in0:band.in1])) for b, f in zip(bufs, fulls))
         q.put((rank, ok))
     finally:
         dist.destroy_process_group()
 
 
 @pytest.mark.parametrize("posted", [False, True])
-@pytest.mark.parametrize("world,H,halo", [(2, 37, 2), (3, 50, 6), (2, 9, 4)])
-def test_exchange_halos_gloo(world, H, halo, posted):
-    """After one exchange every rank holds exactly rows [in0, in1) of the global image."""
+@pytest.mark.parametrize("world,H,halo,n_inputs", [(2, 37, 2, 1), (3, 50, 6, 1), (2, 9, 4, 1), (2, 37, 2, 2),
+                                                   (3, 50, 3, 3)])
+def test_exchange_halos_gloo(world, H, halo, n_inputs, posted):
+    """After one exchange every rank holds exactly rows [in0, in1) of every global
+    input image (multi-input pipelines exchange each input's halo rows)."""
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, H, 23, halo, q, posted)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, H, 23, halo, q, posted, n_inputs))
+             for r in range(world)]
     for p in procs:
         p.start()
     res = dict(q.get(timeout=120) for _ in procs)

@@ -1,0 +1,110 @@
+"""Pre-compiles (NVRTC, no GPU needed) the fused kernels the GPU test suite and
+the bench will launch, into the in-tree cubin cache (paper_conf_cgo_qiaorht19_b200/
+kcache/, keyed by source hash), so that a fresh GPU box only loads modules.
+Runs the compiles in parallel processes.  Scratch tooling, not the product.
+
+    python tools/warm_test_cache.py [-j N]
+"""
+import argparse
+import os
+import random
+import sys
+from multiprocessing import Pool
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def jobs():
+    from kf_inputs import pipelines as P
+    out = []   # (spec, kind, options, hooks)
+    for wl in ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10"]:
+        for size in [(67, 41), (256, 256)]:
+            for kind in ("unfused", "paper", "b200"):
+                out.append((P.WORKLOADS[wl](*size), kind, None, False))
+    for wl in ["harris", "deep10"]:
+        for mode in P.MODES:
+            out.append((P.WORKLOADS[wl](45, 37, mode=mode), "b200", None, False))
+    for size in [(1, 1), (2, 3), (3, 2), (5, 5), (31, 9), (33, 17), (7, 70)]:
+        for wl in ["harris", "deep10", "unsharp"]:
+            for mode in P.MODES:
+                out.append((P.WORKLOADS[wl](*size, mode=mode), "b200", None, False))
+    for seed in range(60):
+        rng = random.Random(70000 + seed)
+        dtype = rng.choice(["f32", "u8x4"])
+        W, H = rng.choice([(1, 1), (4, 3), (9, 9), (33, 17), (70, 45), (129, 20)])
+        spec = P.random_pipeline(rng, W, H, dtype, rng.randint(2, 8))
+        for kind in ("unfused", "paper", "b200"):
+            out.append((spec, kind, None, False))
+    for seed in range(40):
+        rng = random.Random(91000 + seed)
+        dtype = rng.choice(["f32", "u8x4"])
+        W, H = rng.choice([(512, 70), (516, 33), (1024, 41), (640, 131), (2048, 24), (513, 37)])
+        spec = P.random_pipeline(rng, W, H, dtype, rng.randint(2, 6), max_radius=4, asym=0.4)
+        for kind in ("unfused", "paper", "b200"):
+            out.append((spec, kind, None, False))
+    for cfg in ["C1", "C2", "C3", "C3s", "C4", "C5"]:
+        spec, _ = P.config(cfg)
+        for kind in ("unfused", "paper", "b200", "basic"):
+            out.append((spec, kind, None, False))
+    for wl in ["sobel", "enhance"]:
+        for kind in ("unfused", "paper", "b200", "basic"):
+            out.append((P.WORKLOADS[wl](2048, 2048), kind, None, False))
+    same = [{"qptr": 0}, {"lds_pf": 0}, {"const_w": 0}, {"heavy_first": 0}, {"pro_rp": 0}, {"smem_rows": 6},
+            {"sring": 0}, {"minctas": 8}, {"code_budget": 1000}, {"swring": 0}, {"pairs": 0}, {"defer": 0}]
+    exp = [{"v8": 1}, {"persist": 1}, {"nlong": 3}]
+    for wl in ["harris", "deep10", "unsharp"]:
+        for o in same:
+            out.append((P.WORKLOADS[wl](200, 150), "b200", o, False))
+        for o in exp:
+            out.append((P.WORKLOADS[wl](200, 150), "b200", o, True))
+    for mode in ("clamp", "constant"):
+        out.append((P.fig4(mode), "whole", {"naive_border": 1}, True))
+        out.append((P.harris(8, 8, mode), "whole", {"naive_border": 1}, True))
+        out.append((P.fig4(mode), "whole", None, False))
+        out.append((P.harris(8, 8, mode), "whole", None, False))
+    for wl in ["harris", "deep10", "two_input"]:
+        out.append((P.WORKLOADS[wl](96, 130), "b200", None, False))
+    return out
+
+
+def _mod(hooks):
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+    if not hooks:
+        return K
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("kfuse_testhooks", K.__file__)
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    m.lib = m._open(os.path.join(os.path.dirname(K.__file__), "libkfuse_testhooks.so"))
+    return m
+
+
+def compile_job(job):
+    spec, kind, opts, hooks = job
+    K = _mod(hooks)
+    try:
+        p = K.Pipeline.from_spec(spec, opts)
+        plan = (p.plan_unfused() if kind == "unfused" else p.plan_from_blocks([0] * len(spec["ops"]))
+                if kind == "whole" else p.plan_basic("paper") if kind == "basic" else p.plan_fusion(kind))
+        plan.compile()
+        return None
+    except Exception as e:   # noqa: BLE001
+        return f"{spec['name']} {spec['width']}x{spec['height']} {kind} {opts}: {str(e)[:300]}"
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("-j", type=int, default=os.cpu_count())
+    a = ap.parse_args()
+    js = jobs()
+    with Pool(a.j) as pool:
+        errs = [e for e in pool.imap_unordered(compile_job, js, chunksize=1) if e]
+    print(f"{len(js)} plans compiled, {len(errs)} failures")
+    for e in errs:
+        print("FAIL", e)
+    sys.exit(1 if errs else 0)
+
+
+if __name__ == "__main__":
+    main()
