@@ -8,12 +8,17 @@
 N=1: workload C3 = Harris 4096x4096 float32 (clamp), the B200-profile plan
 (fully fused, one launch per step).  A step = one kf_run over one image, inputs
 already resident in HBM; 4 rotating input/output buffer sets (512 MiB > the
-126 MB L2) so consecutive steps never hit in L2.  The unfused (9 launches) and
-paper-profile (6 launches) plans are timed the same way and reported beside it.
-N>1 (torchrun): weak scaling by row bands, each rank a 4096x4096 band of a
-(4096N)x4096 image; every step = one NCCL halo-row exchange + kf_run_band.
---impl reference: the unfused CPU oracle (oracle/) timed on the host cores.
-One JSON line on stdout (rank 0).
+126 MB L2) so consecutive steps never hit in L2.  Every plan (unfused, basic
+[12], paper profile, B200 profile) is timed the same way, and so are the other
+BASELINE configs (C1, C2, C3s, C4, C5 at one GPU) and Sobel / Enhance at 2048^2
+(the paper's Table I shape) under "workloads".
+N>1 (torchrun): the headline is weak scaling by row bands -- each rank a
+4096x4096 band of a (4096N)x4096 image -- and "strong_c5" adds BASELINE C5
+(one 16384x16384 Harris image, 16384/N rows per GPU).  Every step exchanges
+the R halo rows with the neighbours (peer-memory pull over NVLink, or NCCL
+send/recv) behind the band's core rows, then computes the edge strips.
+--impl reference: the unfused CPU oracle (oracle/) timed on the host cores on
+the headline's full image.  One JSON line on stdout (rank 0).
 """
 from __future__ import annotations
 
@@ -33,15 +38,51 @@ import numpy as np  # noqa: E402
 METRIC = "Harris 4096² Mpixel/s fused vs unfused; DRAM bytes/pixel; HBM GB/s vs peak"
 UNIT = "Mpixel/s"
 DATA = "synthetic: counter-based SplitMix64 uniform [0,1) images (kf_inputs/gen.py), as the paper's random images"
-# algorithmic DRAM bytes per pixel of each plan: every launched kernel
-# reads its external inputs once and writes its output once (f32: 4 B per image)
-ALG_BYTES = {"harris": {"unfused": 84, "basic": 60, "paper": 60, "b200": 8},
-             "shitomasi": {"unfused": 84, "basic": 60, "paper": 60, "b200": 8},
-             "unsharp": {"unfused": 44, "basic": 44, "paper": 8, "b200": 8},
-             "deep10": {"unfused": 100, "basic": 92, "paper": 92, "b200": 8}}
 PLANS = ("unfused", "basic", "paper", "b200")
-# the other BASELINE.json configs, timed beside the headline (parity cases otherwise)
-EXTRA_CONFIGS = ("C1", "C2", "C3s", "C4")
+# the other BASELINE.json configs, timed beside the headline (parity cases otherwise),
+# and the paper's Sobel / Enhancement apps at its 2048^2 size (Table I shape)
+EXTRA_CONFIGS = ("C1", "C2", "C3s", "C4", "C5", "sobel:2048", "enhance:2048")
+# context only: the paper's own results on GTX745 / GTX680 / K20c (not targets)
+CONTEXT = {"paper_geomean_speedup_max": 2.52, "paper_geomean_speedup_max_app": "Unsharp",
+           "paper_harris_geomean_speedup": 1.208,
+           "source": "PAPER.md:25-26, 1473-1481 (optimized vs baseline, three Nvidia GPUs)",
+           "note": "fusion vs unfused on other hardware; compare with fused_vs_unfused here, not with value"}
+
+
+def alg_bytes_per_px(spec: dict, blocks) -> int:
+    """Algorithmic DRAM bytes per pixel of a plan: every launched
+    block kernel reads each external image once and writes its sink once (4 B per
+    pixel per image for f32 and for u8x4); halo re-reads excluded."""
+    n_in, ops = spec["n_inputs"], spec["ops"]
+    tot = 0
+    for ks in blocks:
+        inside = {n_in + k for k in ks}
+        ext = {i for k in ks for i in ops[k]["inputs"] if i not in inside}
+        tot += 4 * len(ext) + 4
+    return tot
+
+
+def workload_spec(cfg: str):
+    """A BASELINE config name (C1..C5), or workload:size for a square extra app."""
+    from kf_inputs import pipelines as P
+    if ":" in cfg:
+        wl, n = cfg.split(":")
+        return P.WORKLOADS[wl](int(n), int(n)), 7
+    return P.config(cfg)
+
+
+def host_cpu() -> dict:
+    """nproc and the lscpu model of this host (the CPU baseline's machine)."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "model": model}
 
 
 def load_peaks() -> dict:
@@ -140,39 +181,45 @@ class ClockSampler:
 # ----------------------------------------------------------------- reference
 
 
-def cpu_oracle_run(workload: str, width: int, rows: int, seed: int) -> tuple[float, int]:
-    """Times the unfused oracle on a width x rows image; returns (seconds, pixels)."""
+def cpu_oracle_run(spec: dict, seed: int, threads: int, rows: int | None = None) -> tuple[float, int, int]:
+    """Times the unfused oracle on the workload (or its first `rows` rows as a
+    smaller image of the same width); returns (seconds, pixels, threads used)."""
     from kf_inputs import gen
     from kf_inputs import pipelines as P
     from oracle import oracle as O
-    spec = P.WORKLOADS[workload](width, rows)
-    ins = [gen.image(spec["dtype"], seed, width, rows)]
+    if rows is not None and rows < spec["height"]:
+        spec = P.WORKLOADS[spec["name"]](spec["width"], rows)
+    used = O.set_threads(threads)
+    ins = [gen.image(spec["dtype"], seed + 101 * j, spec["width"], spec["height"]) for j in range(spec["n_inputs"])]
     t = time.perf_counter()
     O.run(spec, ins)
-    return time.perf_counter() - t, width * rows
+    return time.perf_counter() - t, spec["width"] * spec["height"], used
 
 
-def run_reference(args, cfg_name, spec) -> None:
+def run_reference(args, cfg_name, spec, seed) -> None:
+    """The reference arm: the unfused fp64 oracle on ALL host cores (OpenMP over
+    rows), each step one whole image of the headline workload (same config)."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    rows = 128 if spec["dtype"] == "f32" else 32
     for _ in range(args.warmup):
-        cpu_oracle_run(spec["name"], spec["width"], rows, 1)
-    tot, px = 0.0, 0
+        cpu_oracle_run(spec, seed, 0)
+    tot, px, used = 0.0, 0, 1
     for _ in range(args.steps):
-        dt, n = cpu_oracle_run(spec["name"], spec["width"], rows, 1)
+        dt, n, used = cpu_oracle_run(spec, seed, 0)
         tot += dt
         px += n
     v = px / tot / 1e6
-    sample = f"{spec['width']}x{rows} strip of the {spec['width']}x{spec['height']} {spec['name']} workload per step"
+    sample = f"the whole {spec['width']}x{spec['height']} {spec['name']} image per step (same config as the GPU arm)"
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": round(v, 4), "unit": UNIT, "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(tot / args.steps * 1e3, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
         "data": DATA, "config": config_dict(cfg_name, spec, "unfused-oracle", {"l2": "n/a: host oracle"}),
-        "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": round(v, 4), "unit": UNIT, "cores": used, "kind": "oracle", "sample": sample,
+                         "host": host_cpu(), "parallel": "OpenMP over the rows of each kernel"},
         "e2e": {"value": round(v, 4), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "same_config": True,
     }))
 
 
@@ -249,10 +296,10 @@ def bench_single(args, cfg_name, spec, seed) -> None:
             clocks = cs.summary()
         else:
             ms = time_plan(plan, ins, outs, max(50, args.steps // 4), args.warmup, stream, torch)
-        ab = ALG_BYTES.get(spec["name"], {}).get(kind)
+        ab = alg_bytes_per_px(spec, plan.blocks)
         results[kind] = {"ms_per_step": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
                          "launches": plan.num_launches, "alg_bytes_per_px": ab,
-                         "alg_gbs": round(ab * px / (ms * 1e-3) / 1e9, 1) if ab else None}
+                         "alg_gbs": round(ab * px / (ms * 1e-3) / 1e9, 1)}
     head = results[args.plan]
     # distribution over repeated timed replays (the paper reports the median of
     # 500 runs): 11 replays of min(K, 100) steps each, ms/step
@@ -293,12 +340,19 @@ def bench_single(args, cfg_name, spec, seed) -> None:
            "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps}
     if not args.no_extra:
         e2e["pcie_floor"] = pcie_floor(hin, hout, px, torch)
-    # CPU baseline: the unfused oracle on this box's host, one full image
+    # CPU baseline: the unfused oracle on this box's host, one full image, on all
+    # cores (OpenMP over rows) and on one thread (SURVEY §8(d) "two modes")
     cpu = None
     if not args.no_cpu:
-        dt, n = cpu_oracle_run(spec["name"], W, H if spec["dtype"] == "f32" else 256, seed)
-        cpu = {"value": round(n / dt / 1e6, 3), "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"one {W}x{H if spec['dtype'] == 'f32' else 256} image of the workload, unfused fp64 oracle, 1 thread"}
+        rows = None if spec["dtype"] == "f32" else 256
+        dt, n, used = cpu_oracle_run(spec, seed, 0, rows)
+        dt1, n1, _ = cpu_oracle_run(spec, seed, 1, rows)
+        img = f"{W}x{rows or H}"
+        cpu = {"value": round(n / dt / 1e6, 3), "unit": UNIT, "cores": used, "kind": "oracle",
+               "sample": f"one {img} image of the workload, unfused fp64 oracle, OpenMP over rows on {used} threads",
+               "host": host_cpu(),
+               "single_thread": {"value": round(n1 / dt1 / 1e6, 3), "unit": UNIT, "cores": 1,
+                                 "sample": f"the same {img} image, 1 thread"}}
     del ins, outs
     extra = {} if args.no_extra else bench_extra(args, stream, torch, clocks)
     out = {
@@ -310,6 +364,7 @@ def bench_single(args, cfg_name, spec, seed) -> None:
         "gpu_launches": args.steps * hplan.num_launches, "clocks": clocks,
         "plans": results,
         "fused_vs_unfused": round(results["unfused"]["ms_per_step"] / head["ms_per_step"], 3),
+        "context": CONTEXT,
         "workloads": extra,
     }
     print(json.dumps(out))
@@ -373,7 +428,7 @@ def bench_extra(args, stream, torch, clocks) -> dict:
     n_sm = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
     res = {}
     for cfg in EXTRA_CONFIGS:
-        spec, seed = P.config(cfg)
+        spec, seed = workload_spec(cfg)
         W, H = spec["width"], spec["height"]
         px = W * H
         host = gen.image(spec["dtype"], seed, W, H)
@@ -387,14 +442,16 @@ def bench_extra(args, stream, torch, clocks) -> dict:
             p = K.Pipeline.from_spec(spec)
             plan = make_plan(p, kind)
             plan.prepare()
-            steps = 20 if px > 2e7 else 100
+            steps = 6 if px > 1e8 else 20 if px > 2e7 else 100
             ms = time_plan(plan, ins, outs, steps, 3, stream, torch)
-            ab = ALG_BYTES.get(spec["name"], {}).get(kind)
+            ab = alg_bytes_per_px(spec, plan.blocks)
             d["plans"][kind] = {"ms_per_step": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
-                                "launches": plan.num_launches, "alg_bytes_per_px": ab,
-                                "hbm_frac": round(ab * px / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4) if ab else None}
+                                "launches": plan.num_launches, "blocks": len(plan.blocks), "alg_bytes_per_px": ab,
+                                "hbm_frac": round(ab * px / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"], 4)}
         f = d["plans"]["b200"]
         d["fused_vs_unfused"] = round(d["plans"]["unfused"]["ms_per_step"] / f["ms_per_step"], 3)
+        d["basic_vs_unfused"] = round(d["plans"]["unfused"]["ms_per_step"] / d["plans"]["basic"]["ms_per_step"], 3)
+        d["paper_vs_unfused"] = round(d["plans"]["unfused"]["ms_per_step"] / d["plans"]["paper"]["ms_per_step"], 3)
         if px >= 1 << 22:
             d["copy_floor"] = copy_floor(W, H, ins, stream, torch, 8 * px)
             d["copy_floor"]["fused_over_copy"] = round(d["copy_floor"]["ms_per_step"] / f["ms_per_step"], 4)
@@ -407,41 +464,18 @@ def bench_extra(args, stream, torch, clocks) -> dict:
                           "source": "profiles/ncu_inst.json (ncu smsp__inst_executed.sum / px)"}
         res[cfg] = d
         del ins, outs
+        torch.cuda.empty_cache()
     return res
 
 
-def bench_multi(args, cfg_name, spec, seed) -> None:
-    import torch
-    import torch.distributed as dist
-
+def _band_run(args, gspec, seed, plan, rank, world, dev, torch, dist, KD, stream, side, e2e=False) -> dict:
+    """Times `args.steps` row-band steps of one global image on this rank: the
+    halo exchange with the neighbours behind the band's core rows, then the edge
+    strips.  Returns the per-rank timing (max over ranks), the transport, the
+    halo bytes and an exchange-free compute-only time (the same band computed
+    from pre-filled halo rows) that tells whether the exchange was hidden."""
     from kf_inputs import gen
-    from kf_inputs import pipelines as P
-    from paper_conf_cgo_qiaorht19_b200 import dist as KD
-    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
-
-    # KFUSE_DIST_BACKEND=gloo and KFUSE_BENCH_DEVICE=0 let a 2-rank smoke run share one GPU (tests only)
-    dist.init_process_group(os.environ.get("KFUSE_DIST_BACKEND", "nccl"))
-    rank, world = dist.get_rank(), dist.get_world_size()
-    dev = int(os.environ.get("KFUSE_BENCH_DEVICE", os.environ.get("LOCAL_RANK", rank)))
-    torch.cuda.set_device(dev)
-    # NCCL prints its version banner on stdout when the first communicator is
-    # created: create it now with stdout pointed at stderr (stdout carries the
-    # one JSON line)
-    sys.stdout.flush()
-    saved = os.dup(1)
-    os.dup2(2, 1)
-    try:
-        dist.barrier()
-    finally:
-        sys.stdout.flush()
-        os.dup2(saved, 1)
-        os.close(saved)
-    W, Hb = spec["width"], spec["height"]
-    Htot = Hb * world                                 # weak scaling: one band per GPU
-    gspec = P.WORKLOADS[spec["name"]](W, Htot)
-    p = K.Pipeline.from_spec(gspec)
-    plan = make_plan(p, args.plan)
-    plan.prepare()
+    W, Htot = gspec["width"], gspec["height"]
     band = KD.partition(Htot, world, rank, plan.halo_rows)
     host = gen.image(gspec["dtype"], seed, W, Htot, band.in0, band.in1)
     tdt = torch.float32 if gspec["dtype"] == "f32" else torch.uint8
@@ -449,9 +483,6 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
     ins = [torch.from_numpy(host).cuda() for _ in range(nsets)]
     oshape = (band.rows, W) if gspec["dtype"] == "f32" else (band.rows, W, 4)
     outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(nsets)]
-    stream = torch.cuda.Stream()
-    torch.cuda.set_stream(stream)
-    side = torch.cuda.Stream()
     # halo transport: peer memory (CUDA IPC mappings over NVLink, device-counter
     # sync, whole steps captured in a CUDA graph) or NCCL send/recv (eager)
     mode = os.environ.get("KFUSE_HALO", "peer")
@@ -467,6 +498,9 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
         dist.all_reduce(agree, op=dist.ReduceOp.MIN)
         if int(agree.item()) == 0 and mode == "peer":
             mode, halo, note = "nccl", None, "peer setup failed on another rank; "
+    ref_out = torch.empty_like(outs[0])
+    plan.run_band(band.row0, band.row1, [ins[0]], band.in0, band.in1, [ref_out], stream)
+    torch.cuda.synchronize()
     if mode == "peer" and (halo.up is not None or halo.down is not None):
         # Self-check on this hardware before timing: the buffers were generated
         # with their halo rows, so kf_run_band over them is the reference.  Poison
@@ -474,9 +508,6 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
         # rank falls back to NCCL (and says so in the JSON line).
         ok = 1
         try:
-            ref_out = torch.empty_like(outs[0])
-            plan.run_band(band.row0, band.row1, [ins[0]], band.in0, band.in1, [ref_out], stream)
-            torch.cuda.synchronize()
             t_, n_ = band.top, band.rows
             if gspec["dtype"] == "f32":
                 ins[0][:t_].fill_(float("nan"))
@@ -498,8 +529,9 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
             mode, halo, note = "nccl", None, note + "peer self-check failed; "
             ins[0].copy_(torch.from_numpy(host).to(ins[0].device))   # restore the halo rows
     (c0, c1), edges = KD.split_rows(band)
-    exch = halo is not None and (halo.up is not None or halo.down is not None)
-    launches_per_step = plan.num_launches * ((1 if c1 > c0 else 0) + len(edges)) + (2 if exch else 0)
+    exch = world > 1 and plan.halo_rows > 0 and (halo is None or halo.up is not None or halo.down is not None)
+    launches_per_step = plan.num_launches * ((1 if c1 > c0 else 0) + len(edges)) + \
+        (2 if exch and mode == "peer" else 0)
 
     def step(i):
         if mode == "peer":   # core rows || (signal, halo pull over peer loads), then the edge strips
@@ -507,95 +539,184 @@ def bench_multi(args, cfg_name, spec, seed) -> None:
         else:                # NCCL send/recv overlapped with the core rows
             KD.run_step_overlapped(plan, band, [ins[i % nsets]], [outs[i % nsets]], side)
 
-    for i in range(args.warmup):
-        step(i)
-    torch.cuda.synchronize()
-    graph = None
-    if mode == "peer":   # every rank captures the same steps; the counters synchronise the replays
-        graph = torch.cuda.CUDAGraph()
-        with torch.cuda.graph(graph, stream=stream):
-            for i in range(args.steps):
-                step(i)
+    def timed(fn, graphable):
+        for i in range(args.warmup):
+            fn(i)
         torch.cuda.synchronize()
+        graph = None
+        if graphable:   # every rank captures the same steps; the counters synchronise the replays
+            graph = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(graph, stream=stream):
+                for i in range(args.steps):
+                    fn(i)
+            torch.cuda.synchronize()
+            dist.barrier()
+            with torch.cuda.stream(stream):   # one untimed replay: the first launch uploads the graph
+                graph.replay()
+            torch.cuda.synchronize()
         dist.barrier()
-        with torch.cuda.stream(stream):   # one untimed replay: the first launch uploads the graph
-            graph.replay()
-        torch.cuda.synchronize()
-    dist.barrier()
-    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(dev) as cs:
-        t0.record(stream)
-        if graph is not None:
-            graph.replay()
-        else:
-            for i in range(args.steps):
-                step(i)
-        t1.record(stream)
-        torch.cuda.synchronize()
-    dist.barrier()
-    ms = torch.tensor([t0.elapsed_time(t1) / args.steps], device="cuda")
-    dist.all_reduce(ms, op=dist.ReduceOp.MAX)
-    ms = float(ms.item())
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with ClockSampler(dev) as cs:
+            t0.record(stream)
+            if graph is not None:
+                graph.replay()
+            else:
+                for i in range(args.steps):
+                    fn(i)
+            t1.record(stream)
+            torch.cuda.synchronize()
+        dist.barrier()
+        ms = torch.tensor([t0.elapsed_time(t1) / args.steps], device="cuda")
+        dist.all_reduce(ms, op=dist.ReduceOp.MAX)
+        del graph
+        return float(ms.item()), cs.summary()
+
+    ms, clocks = timed(step, mode == "peer")
     if halo is not None:
         bad = torch.tensor([halo.errors()], device="cuda")
         dist.all_reduce(bad, op=dist.ReduceOp.MAX)
         if int(bad.item()):
             raise RuntimeError("peer halo: a counter wait timed out")
-    px = W * Htot
-    # end to end through the public API: each step uploads the band's own rows
-    # from pinned host memory, runs the step (halo exchange + fused kernels) and
-    # downloads the band's output; max over ranks of the wall time
-    hin = torch.from_numpy(host).pin_memory()
-    hout = torch.empty(oshape, dtype=tdt).pin_memory()
-    t, n = band.top, band.rows
-    e2e_steps = max(3, min(args.steps, 20))
+    # the same band work without any exchange (halo rows already in place): if
+    # the step costs no more than this, the exchange was hidden behind the core
+    for k in range(nsets):
+        ins[k].copy_(torch.from_numpy(host).to(ins[k].device))
 
-    def e2e_step():
-        if halo is not None:
-            halo.wait_consumed(stream)        # the neighbours pulled the previous rows
-        ins[0][t:t + n].copy_(hin[t:t + n], non_blocking=True)
-        if halo is not None:
-            halo.step(plan, 0, [outs[0]], stream, side)
-        else:
-            KD.run_step_overlapped(plan, band, [ins[0]], [outs[0]], side)
-        hout.copy_(outs[0], non_blocking=True)
-        stream.synchronize()
+    def compute_only(i):
+        plan.run_band(band.row0, band.row1, [ins[i % nsets]], band.in0, band.in1, [outs[i % nsets]], stream)
+    ms_c, _ = timed(compute_only, True)
+    rb = W * 4
+    halo_bytes = (band.top + band.bottom) * rb * gspec["n_inputs"] if exch else 0
+    hb = torch.tensor([halo_bytes], dtype=torch.float64, device="cuda")
+    dist.all_reduce(hb, op=dist.ReduceOp.SUM)
+    res = {"ms": ms, "clocks": clocks, "mode": mode, "note": note, "band": band, "plan": plan,
+           "launches_per_step": launches_per_step,
+           "exchange": {"transport": ("peer-memory halo pull (CUDA IPC / NVLink P2P, device-counter sync), steps "
+                                      "replayed from a CUDA graph") if mode == "peer" else
+                        "NCCL send/recv overlapped with the core rows",
+                        "halo_rows": plan.halo_rows, "halo_bytes_per_step_this_rank": halo_bytes,
+                        "halo_bytes_per_step_all_ranks": int(hb.item()),
+                        "step_ms": round(ms, 5), "compute_only_ms": round(ms_c, 5),
+                        "exchange_overhead_frac": round(ms / ms_c - 1.0, 4),
+                        "hidden": bool(ms <= ms_c * 1.03)}}
+    if e2e:
+        # end to end through the public API: each step uploads the band's own rows
+        # from pinned host memory, runs the step (halo exchange + fused kernels)
+        # and downloads the band's output; max over ranks of the wall time
+        hin = torch.from_numpy(host).pin_memory()
+        hout = torch.empty(oshape, dtype=tdt).pin_memory()
+        t, n = band.top, band.rows
+        e2e_steps = max(3, min(args.steps, 20))
 
-    e2e_step()
-    dist.barrier()
-    tw = time.perf_counter()
-    for _ in range(e2e_steps):
+        def e2e_step():
+            if halo is not None:
+                halo.wait_consumed(stream)        # the neighbours pulled the previous rows
+            ins[0][t:t + n].copy_(hin[t:t + n], non_blocking=True)
+            if halo is not None:
+                halo.step(plan, 0, [outs[0]], stream, side)
+            else:
+                KD.run_step_overlapped(plan, band, [ins[0]], [outs[0]], side)
+            hout.copy_(outs[0], non_blocking=True)
+            stream.synchronize()
+
         e2e_step()
-    e2e_s = torch.tensor([(time.perf_counter() - tw) / e2e_steps], device="cuda")
-    dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX)
-    e2e = {"value": round(px / float(e2e_s.item()) / 1e6, 1), "unit": UNIT,
-           "h2d_bytes_per_step": int(n * hin[0].numel() * hin.element_size()),
-           "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps,
-           "note": "per rank, max over ranks"}
-    how = ("peer-memory halo pull (CUDA IPC / NVLink P2P, device-counter sync), steps replayed from a CUDA graph"
-           if mode == "peer" else "NCCL send/recv overlapped with the core rows")
-    if rank == 0:
-        ab = ALG_BYTES.get(gspec["name"], {}).get(args.plan) or 8
-        peaks = load_peaks()
-        ach = ab * (band.rows * W) / (ms * 1e-3) / 1e9
-        print(json.dumps({
-            "metric": METRIC, "value": round(px / (ms * 1e-3) / 1e6, 1), "unit": UNIT, "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": DATA,
-            "config": config_dict(cfg_name, gspec, args.plan,
-                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows: {note}{how}",
-                                   "band": f"{Hb}x{W} per GPU"}),
-            "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                         "frac": round(ach / peaks["hbm_gbs"], 4), "traffic": None,
-                         "peak_source": peaks["source"], "note": "per GPU, step time incl. halo exchange"},
-            "cpu_baseline": None,
-            "e2e": e2e,
-            "gpu_launches": args.steps * launches_per_step, "clocks": cs.summary(),
-        }))
+        dist.barrier()
+        tw = time.perf_counter()
+        for _ in range(e2e_steps):
+            e2e_step()
+        e2e_s = torch.tensor([(time.perf_counter() - tw) / e2e_steps], device="cuda")
+        dist.all_reduce(e2e_s, op=dist.ReduceOp.MAX)
+        res["e2e"] = {"value": round(W * Htot / float(e2e_s.item()) / 1e6, 1), "unit": UNIT,
+                      "h2d_bytes_per_step": int(n * hin[0].numel() * hin.element_size()),
+                      "d2h_bytes_per_step": int(hout.numel() * hout.element_size()), "steps": e2e_steps,
+                      "note": "per rank, max over ranks"}
     if halo is not None:   # drop the peer mappings on every rank before any rank frees its buffers
         halo.close()
         dist.barrier()
-    del graph
+    res["_keep"] = (halo, ins, outs)   # freed by the caller after every rank is done
+    return res
+
+
+def bench_multi(args, cfg_name, spec, seed) -> None:
+    import torch
+    import torch.distributed as dist
+
+    from kf_inputs import pipelines as P
+    from paper_conf_cgo_qiaorht19_b200 import dist as KD
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+
+    # KFUSE_DIST_BACKEND=gloo and KFUSE_BENCH_DEVICE=0 let a 2-rank smoke run share one GPU (tests only)
+    dist.init_process_group(os.environ.get("KFUSE_DIST_BACKEND", "nccl"))
+    rank, world = dist.get_rank(), dist.get_world_size()
+    dev = int(os.environ.get("KFUSE_BENCH_DEVICE", os.environ.get("LOCAL_RANK", rank)))
+    torch.cuda.set_device(dev)
+    # NCCL prints its version banner on stdout when the first communicator is
+    # created: create it now with stdout pointed at stderr (stdout carries the
+    # one JSON line)
+    sys.stdout.flush()
+    saved = os.dup(1)
+    os.dup2(2, 1)
+    try:
+        dist.barrier()
+    finally:
+        sys.stdout.flush()
+        os.dup2(saved, 1)
+        os.close(saved)
+    stream = torch.cuda.Stream()
+    torch.cuda.set_stream(stream)
+    side = torch.cuda.Stream()
+    peaks = load_peaks()
+    dtype = "f32" if spec["dtype"] == "f32" else "u8x4/int32"
+
+    # headline: weak scaling, one band of the config's size per GPU
+    W, Hb = spec["width"], spec["height"]
+    gspec = P.WORKLOADS[spec["name"]](W, Hb * world)
+    plan = make_plan(K.Pipeline.from_spec(gspec), args.plan)
+    plan.prepare()
+    weak = _band_run(args, gspec, seed, plan, rank, world, dev, torch, dist, KD, stream, side, e2e=True)
+    # BASELINE C5: one 16384^2 Harris image split into `world` bands (strong scaling)
+    strong = None
+    if not args.no_extra and cfg_name != "C5":
+        c5, c5seed = P.config("C5")
+        c5plan = make_plan(K.Pipeline.from_spec(c5), args.plan)
+        c5plan.prepare()
+        strong = _band_run(args, c5, c5seed, c5plan, rank, world, dev, torch, dist, KD, stream, side)
+
+    def summary(r, g):
+        px_all = g["width"] * g["height"]
+        band = r["band"]
+        ab = alg_bytes_per_px(g, r["plan"].blocks)
+        ach = ab * (band.rows * g["width"]) / (r["ms"] * 1e-3) / 1e9
+        return px_all, {"bound": "hbm", "achieved": round(ach, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                        "frac": round(ach / peaks["hbm_gbs"], 4), "traffic": None,
+                        "peak_source": peaks["source"], "note": "per GPU (largest band), step time incl. halo exchange"}
+
+    if rank == 0:
+        px, roof = summary(weak, gspec)
+        out = {
+            "metric": METRIC, "value": round(px / (weak["ms"] * 1e-3) / 1e6, 1), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(weak["ms"], 5),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": dtype, "data": DATA,
+            "config": config_dict(cfg_name, gspec, args.plan,
+                                  {"parallelism": f"row bands x{world}, halo {plan.halo_rows} rows: "
+                                                  f"{weak['note']}{weak['exchange']['transport']}",
+                                   "band": f"{Hb}x{W} per GPU"}),
+            "roofline": roof, "cpu_baseline": None, "e2e": weak["e2e"],
+            "gpu_launches": args.steps * weak["launches_per_step"], "clocks": weak["clocks"],
+            "exchange": weak["exchange"], "context": CONTEXT,
+        }
+        if strong is not None:
+            c5, _ = P.config("C5")
+            px5, roof5 = summary(strong, c5)
+            out["strong_c5"] = {
+                "workload": f"C5: harris {c5['width']}x{c5['height']} f32, {world} row bands", "scaling": "strong",
+                "value": round(px5 / (strong["ms"] * 1e-3) / 1e6, 1), "unit": UNIT,
+                "ms_per_step": round(strong["ms"], 5), "rows_per_gpu": strong["band"].rows,
+                "roofline": roof5, "exchange": strong["exchange"],
+                "gpu_launches": args.steps * strong["launches_per_step"]}
+        print(json.dumps(out))
+    dist.barrier()
+    del weak, strong
     torch.cuda.synchronize()
     dist.destroy_process_group()
     # Leave without the interpreter's teardown: torch's CUDA-IPC bookkeeping of
@@ -622,7 +743,7 @@ def main():
     from kf_inputs import pipelines as P
     spec, seed = P.config(args.config)
     if args.impl == "reference":
-        run_reference(args, args.config, spec)
+        run_reference(args, args.config, spec, seed)
         return
     world = int(os.environ.get("WORLD_SIZE", "1"))
     if world > 1 or args.force_multi:

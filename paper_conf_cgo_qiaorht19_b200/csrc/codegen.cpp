@@ -957,6 +957,7 @@ struct StreamGen {
     bool defer_ok = true;  // pair mode: defer normalised masks' power-of-two scales (option "defer")
     std::set<int> prp;     // external images fed by running row pointers from the prologue on (interior strips)
     bool qptr = false;     // steady-state loop: ring slots addressed from per-trip base pointers
+    bool tma = false;      // this variant feeds the ring with TMA bulk row copies (option tma)
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp},
@@ -1543,16 +1544,41 @@ struct StreamGen {
                                        << (k ? " + " + std::to_string(4 * k) : "") << ");";
         o << " }\n";
     }
+    // mbarrier of ring slot `ss` of image slot s (TMA feed)
+    std::string bar(int s, const std::string &ss) const
+    {
+        return "(mb + " + std::to_string(s * si.DS) + " + (" + ss + "))";
+    }
+    // TMA feed: lane 0 copies the warp's whole row segment (tb bytes) with one bulk copy
+    void bulk_row(const std::string &dst, const std::string &src, const std::string &guard, int s,
+                  const std::string &ss, const std::string &ind)
+    {
+        o << ind << "if (lane == 0 && " << guard << ") kf_bulk_row((char *)(" << dst << ") + toff, " << src << ", tb, "
+          << bar(s, ss) << ");\n";
+    }
     void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
     {
         int s = slot.at(img);
         if (runptr || prp.count(img)) {   // running row pointer (rows stay inside [base, rlast])
-            cp_row(slot_ptr(s, ss), "ip" + std::to_string(s), "(" + it + ") < nit", ind);
+            if (tma)
+                bulk_row(slot_ptr(s, ss), "ip" + std::to_string(s), "(" + it + ") < nit", s, ss, ind);
+            else
+                cp_row(slot_ptr(s, ss), "ip" + std::to_string(s), "(" + it + ") < nit", ind);
             o << ind << "ip" << s << " += dW;\n";
             return;
         }
         std::string row = row_of(img, it, ind);
-        cp_row(slot_ptr(s, ss), "g" + std::to_string(s) + " + " + row + " * W", "(" + it + ") < nit", ind);
+        if (tma)
+            bulk_row(slot_ptr(s, ss), "g" + std::to_string(s) + " + " + row + " * W", "(" + it + ") < nit", s, ss, ind);
+        else
+            cp_row(slot_ptr(s, ss), "g" + std::to_string(s) + " + " + row + " * W", "(" + it + ") < nit", ind);
+    }
+    // TMA feed: wait until the row of iteration `it` (ring slot ss, phase parity par) landed
+    void wait_row(const std::string &ss, const std::string &par, const std::string &it, const std::string &ind)
+    {
+        o << ind << "if ((" << it << ") < nit) {";
+        for (int img : b.ext) o << " kf_mbar_wait(" << bar(slot.at(img), ss) << ", " << par << ");";
+        o << " }\n";
     }
     // shared-memory ring: read ring slot `ss` into register ring slot rs
     void fetch(int img, const std::string &ss, int rs, const std::string &ind)
@@ -1588,20 +1614,36 @@ struct StreamGen {
                 s_iss = j == 0 ? "qprev" : "qb + " + std::to_string(j - 1);
                 s_get = "qb + " + std::to_string(j);
             }
+            const std::string row_get = uexpr + " + " + std::to_string(j);
+            const std::string row_nxt = uexpr + " + " + std::to_string(j + 1);
+            if (tma) {   // every lane has read the slot about to be refilled (read a row or two ago)
+                o << ind << "__syncwarp();\n";
+                o << ind << "if (lane == 0) kf_proxy_fence();\n";
+            }
             for (int img : b.ext) issue(img, s_iss, uexpr + " + " + std::to_string(j + DS - 1), ind);
-            o << ind << "kf_cp_commit();\n";
+            if (!tma) o << ind << "kf_cp_commit();\n";
+            // TMA: phase parity of the row's slot = (row / DS) & 1, tracked as `ph` (flips when qb wraps)
+            const std::string p_get = u >= 0 ? std::to_string((u / DS) & 1) : "ph";
             if (si.lpf) {
                 // this iteration's row is already in registers; wait for the next
                 // row and read it now, a whole iteration before its use
                 for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
+                const bool wrap = !(u >= 0) && !(j + 1 < si.P && !si.rolled);
                 const std::string s_nxt = u >= 0 ? std::to_string((u + 1) % DS)
-                                                 : (j + 1 < si.P && !si.rolled ? "qb + " + std::to_string(j + 1) : "qnext");
-                o << ind << "kf_cp_wait<" << DS - 2 << ">();\n";
+                                                 : (!wrap ? "qb + " + std::to_string(j + 1) : "qnext");
+                const std::string p_nxt = u >= 0 ? std::to_string(((u + 1) / DS) & 1) : wrap ? "(ph ^ (qnext == 0))" : "ph";
+                if (tma)
+                    wait_row(s_nxt, p_nxt, row_nxt, ind);
+                else
+                    o << ind << "kf_cp_wait<" << DS - 2 << ">();\n";
                 for (int img : b.ext)
                     for (int k = 0; k < NQ; k++)
                         o << ind << "pf" << slot.at(img) << "_" << k << " = *(" << slot_ptr(slot.at(img), s_nxt) << " + " << k << ");\n";
             } else {
-                o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
+                if (tma)
+                    wait_row(s_get, p_get, row_get, ind);
+                else
+                    o << ind << "kf_cp_wait<" << DS - 1 << ">();\n";
                 for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
             }
         } else {
@@ -1687,6 +1729,9 @@ struct StreamGen {
         dir = dir_;
         el = l;
         er = r;
+        // TMA row feed (option tma): interior chunks only -- an edge chunk clamps
+        // its lanes' columns, so its row segment is not one contiguous copy
+        tma = si.sring && si.vec && si.tma && !l && !r;
         const int P = si.P, D = si.D, L = si.L, HL = si.HL;
         o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast" << vname(dir, ve, l, r)
           << "(const KfArgs &a, const int chunk, const int strip)\n{\n";
@@ -1760,12 +1805,33 @@ struct StreamGen {
                 o << "    " << (f32 ? "float4" : "uint4") << " *sr" << s << " = (" << (f32 ? "float4" : "uint4")
                   << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 * NQ << ") + lane * " << NQ << ";\n";
             }
+            if (tma) {
+                // one mbarrier per (image, ring slot) after the rings.  The warp's
+                // row segment is lanes 0..31's columns [x0w, x0w + 32V) clipped to
+                // the image (W % 4 == 0, x0w % 4 == 0: 16-B multiples); lane 0's row
+                // pointer already starts at the clipped column max(x0w, 0), which
+                // lands at byte toff of the slot.  Lanes wholly outside the image
+                // keep stale ring data: they are halo lanes no stored pixel reads.
+                o << "    unsigned long long *mb = (unsigned long long *)(" << kernel_name(block) << "_smem + "
+                  << si.ring_bytes << ");\n";
+                o << "    const int x0w = a.fx0 + (chunk * " << 32 - 2 * HL << " - " << HL << ") * " << V << ";\n";
+                o << "    const unsigned toff = (unsigned)(max(x0w, 0) - x0w) * 4u;\n";
+                o << "    const unsigned tb = (unsigned)(min(x0w + " << 32 * V << ", W) - max(x0w, 0)) * 4u;\n";
+                o << "    if (lane == 0) {\n";
+                o << "        for (int i = 0; i < " << (int)b.ext.size() * si.DS << "; i++) kf_mbar_init(mb + i, 1);\n";
+                o << "        kf_mbar_init_fence();\n";
+                o << "    }\n";
+                o << "    __syncwarp();\n";
+            }
             for (int it = 0; it < si.DS - 1; it++) {
                 for (int img : b.ext) issue(img, std::to_string(it), std::to_string(it), "    ");
-                o << "    kf_cp_commit();\n";
+                if (!tma) o << "    kf_cp_commit();\n";
             }
             if (si.lpf) {
-                o << "    kf_cp_wait<" << si.DS - 2 << ">();\n";
+                if (tma)
+                    wait_row("0", "0", "0", "    ");
+                else
+                    o << "    kf_cp_wait<" << si.DS - 2 << ">();\n";
                 for (int img : b.ext) {
                     int s = slot.at(img);
                     for (int k = 0; k < NQ; k++)
@@ -1773,6 +1839,7 @@ struct StreamGen {
                 }
             }
             o << "    int qb = 0;   // ring slot of the current iteration's row (multiple of the unroll)\n";
+            if (tma) o << "    unsigned ph = 0;   // phase parity of ring slot qb's current row\n";
         } else {
             for (int it = 0; it < D; it++)
                 for (int img : b.ext) load(img, si.rolled ? D - it : it % P, std::to_string(it), "    ");
@@ -1793,6 +1860,7 @@ struct StreamGen {
             for (int u = 0; u < Q; u++) iteration(u % P, u, std::to_string(u - u % P), "      ");
             u0 = Q;
             if (si.sring) o << "    qb = " << Q % si.DS << ";\n";
+            if (tma) o << "    ph = " << ((Q / si.DS) & 1) << ";\n";
         }
         vedge = false;
         const int step = si.rolled ? 1 : P;
@@ -1834,7 +1902,9 @@ struct StreamGen {
             for (int j = 0; j < P; j++) iteration(j, -1, "u", "        ");
             qptr = false;
         }
-        if (si.sring) o << "        qb += " << step << ";\n        if (qb == " << si.DS << ") qb = 0;\n";
+        if (si.sring)
+            o << "        qb += " << step << ";\n        if (qb == " << si.DS << ") { qb = 0;" << (tma ? " ph ^= 1u;" : "")
+              << " }\n";
         o << "    }\n}\n\n";
         runptr = false;
     }
@@ -1965,8 +2035,8 @@ const OptDef kOpts[] = {
     {"swar", 1, 0, 1, false},           // u8x4 kernels in SWAR form (§5.2b)
     {"swring", 1, 0, 1, false},         // unpacked SWAR rings
     {"swring_cap", 164, 0, 1024, false},
-    {"pairs", 1, 0, 1, false},          // f32 packed pixel pairs (FFMA2/FADD2)
-    {"defer", 1, 0, 1, false},          // deferred power-of-two mask scales
+    {"pairs", 1, 0, 1, true},           // f32 packed pixel pairs (FFMA2/FADD2); off changes rounding
+    {"defer", 1, 0, 1, true},           // deferred power-of-two mask scales; off changes rounding
     {"prefetch", 4, 1, 16, false},      // register prefetch distance (no smem ring)
     {"sring", 1, 0, 1, false},          // cp.async shared-memory row ring
     {"smem_rows", 12, 2, 64, false},    // rows of that ring
@@ -1980,6 +2050,7 @@ const OptDef kOpts[] = {
     {"minctas", kMinCtasPerSm, 1, 32, false},    // __launch_bounds__ min CTAs per SM
     {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)
     {"host_taper", 1, 0, 1, false},     // kf_run_host thin first/last bands
+    {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
     {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
     {"persist_waves", 1, 1, 1 << 20, true},
@@ -2106,6 +2177,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         si.DS = DS;
         si.ring_bytes = (int)b.ext.size() * DS * 128 * kV_;
         si.lpf = si.sring && DS >= 3 && opt(p, "lds_pf");
+        si.tma = si.sring && opt(p, "tma");
     }
     if (!si.sring) si.P = std::max(maxdepth, maxdepth_ext + si.D);
     // register estimate: live ring values (depth per image, D prefetched rows)
@@ -2214,7 +2286,8 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
             n = std::max(n, (kFrameTiles[s][0] + 2 * b.hx.at(k)) * (kFrameTiles[s][1] + 2 * b.hy.at(k)));
         frame_bytes += n * 4;
     }
-    const int smem_bytes = std::max(16, std::max(frame_bytes, si.ok && si.sring ? si.ring_bytes : 0));
+    const int ring_total = si.ring_bytes + (si.tma ? 8 * (int)b.ext.size() * si.DS : 0);   // + TMA mbarriers
+    const int smem_bytes = std::max(16, std::max(frame_bytes, si.ok && si.sring ? ring_total : 0));
     o << "__shared__ __align__(16) unsigned char " << kernel_name(block) << "_smem[" << smem_bytes << "];\n\n";
     FrameGen fg(p, b, block, o);
     fg.run();

@@ -279,4 +279,36 @@ template <int N> __device__ __forceinline__ void kf_cp_wait()
 {
     asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
 }
+
+// ------------------------------------- TMA row feed (option tma)
+// The same ring, filled by the Tensor Memory Accelerator instead: one elected
+// lane issues ONE bulk copy (cp.async.bulk, SASS UBLKCP) of the warp's whole
+// contiguous row segment (32 lanes x 16 B) per row, completing on an mbarrier
+// per ring slot (expect_tx / complete_tx); the lanes wait on the slot's phase
+// parity instead of a cp.async group count.  Before a slot is refilled the
+// warp synchronises (every lane has read it) and the issuing lane orders those
+// generic-proxy reads before the async-proxy write (fence.proxy.async).
+__device__ __forceinline__ unsigned kf_smem_addr(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void kf_mbar_init(unsigned long long *bar, unsigned count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(kf_smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void kf_mbar_init_fence() { asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory"); }
+__device__ __forceinline__ void kf_proxy_fence() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
+__device__ __forceinline__ void kf_bulk_row(void *smem, const void *gmem, unsigned bytes, unsigned long long *bar)
+{
+    const unsigned b = kf_smem_addr(bar);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(b), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
+                 ::"r"(kf_smem_addr(smem)), "l"(gmem), "r"(bytes), "r"(b) : "memory");
+}
+__device__ __forceinline__ void kf_mbar_wait(unsigned long long *bar, unsigned parity)
+{
+    const unsigned b = kf_smem_addr(bar);
+    unsigned done;
+    do {
+        asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+                     : "=r"(done) : "r"(b), "r"(parity) : "memory");
+    } while (!done);
+}
 __device__ __forceinline__ int kf_wrap_lt(int x, int n) { return x >= n ? x - n : x; }

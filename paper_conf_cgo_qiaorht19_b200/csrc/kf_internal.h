@@ -149,6 +149,7 @@ struct StreamInfo {
     bool sring = false;           // external rows fed by a cp.async shared-memory ring
     int DS = 0;                   // rows in that ring (multiple of P)
     bool lpf = false;             // ring rows read one iteration ahead (LDS latency off the critical path)
+    bool tma = false;             // the ring is filled by TMA bulk row copies (option tma)
     int ring_bytes = 0;           // its shared memory per warp
     long long iter_ops = 0;       // scalar operations per iteration (code-size estimate)
     bool edge_v = false;          // top/bottom image edges handled by edge strips

@@ -69,9 +69,9 @@ def check(spec, got, ref, what="", pointwise=True):
 def pointwise_rel(got, ref):
     """max |g - o| / |o| over the pixels with |o| >= PW_FLOOR * max|o|."""
     a = np.abs(ref)
+    if a.max() == 0:    # an all-zero oracle output: the normalised check decides
+        return float(np.abs(got).max())
     sel = a >= PW_FLOOR * a.max()
-    if not sel.any():
-        return 0.0
     return float((np.abs(got.astype(np.float64) - ref)[sel] / a[sel]).max())
 
 
@@ -427,6 +427,13 @@ def _peer_worker(rank, world, port, wl, graph, q):
         dist.barrier()
     finally:
         dist.destroy_process_group()
+    # Leave without the interpreter's teardown (as bench.py does): torch's CUDA-IPC
+    # bookkeeping of the exchanged buffers can crash at exit after every rank has
+    # released them and reported its result.
+    q.close()
+    q.join_thread()
+    import os as _os2
+    _os2._exit(0)
 
 
 @pytest.mark.parametrize("wl,world,graph", [("harris", 2, False), ("harris", 3, True), ("deep10", 2, True),
@@ -475,8 +482,12 @@ def test_strip_geometry_bit_identical(wl):
 # is scheduled: results must stay bit-identical to the default.  The
 # experimental ones (v8, persist, nlong) exist only in the test-hooks build.
 SAME_BITS = [{"qptr": 0}, {"lds_pf": 0}, {"const_w": 0}, {"heavy_first": 0}, {"pro_rp": 0}, {"smem_rows": 6},
-             {"sring": 0}, {"minctas": 8}, {"code_budget": 1000}, {"swring": 0}, {"pairs": 0}, {"defer": 0}]
+             {"sring": 0}, {"minctas": 8}, {"code_budget": 1000}, {"swring": 0}, {"tma": 1},
+             {"tma": 1, "lds_pf": 0}, {"tma": 1, "code_budget": 1000}, {"tma": 1, "smem_rows": 6}]
 EXPERIMENTAL = [{"v8": 1}, {"persist": 1}, {"nlong": 3}, {"persist": 1, "persist_waves": 2}]
+# experimental options that change the f32 rounding (scalar instead of packed pairs,
+# scales applied per stage): within the parity tolerance of the oracle, not bit-identical
+EXPERIMENTAL_ROUNDING = [{"pairs": 0}, {"defer": 0}]
 
 
 def _hooks():
@@ -501,6 +512,16 @@ def test_schedule_options_bit_identical(wl, opts):
     mod = _hooks() if opts in EXPERIMENTAL else None
     got = run_gpu(spec, make_plan(spec, "b200", opts, mod), ins)[0]
     np.testing.assert_array_equal(got, base)
+
+
+@pytest.mark.parametrize("wl", ["harris", "unsharp", "shitomasi"])
+@pytest.mark.parametrize("opts", EXPERIMENTAL_ROUNDING, ids=lambda o: ",".join(f"{k}={v}" for k, v in o.items()))
+def test_experimental_rounding_options_within_tolerance(wl, opts):
+    spec = P.WORKLOADS[wl](200, 150)
+    ins = _inputs(spec, 12)
+    ref = O.run(spec, ins)[spec["outputs"][0]]
+    got = run_gpu(spec, make_plan(spec, "b200", opts, _hooks()), ins)[0]
+    check(spec, got, ref, f"{wl} {opts}")
 
 
 @pytest.mark.parametrize("wl", ["deep10", "harris"])
