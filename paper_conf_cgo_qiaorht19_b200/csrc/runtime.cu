@@ -10,6 +10,7 @@
 #include <dlfcn.h>
 #include <nvrtc.h>
 #include <sys/stat.h>
+#include <utime.h>
 #include <unistd.h>
 
 #include <cstdio>
@@ -120,7 +121,10 @@ static std::string compile_cubin(const std::string &src, const std::string &name
             std::stringstream ss;
             ss << f.rdbuf();
             std::string s = ss.str();
-            if (s.size() > 16) return s;
+            if (s.size() > 16) {
+                utime(path.c_str(), nullptr);   // mark as used (tools/warm_test_cache.py --prune keeps used cubins)
+                return s;
+            }
         }
     }
     nvrtcProgram prog;

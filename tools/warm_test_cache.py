@@ -105,11 +105,20 @@ def compile_job(job):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("-j", type=int, default=os.cpu_count())
+    ap.add_argument("--prune", action="store_true", help="delete cached cubins this warm-up did not use")
     a = ap.parse_args()
+    import time
+    t0 = time.time() - 2
     js = jobs()
     with Pool(a.j) as pool:
         errs = [e for e in pool.imap_unordered(compile_job, js, chunksize=1) if e]
     print(f"{len(js)} plans compiled, {len(errs)} failures")
+    if a.prune and not errs:
+        cache = os.path.join(ROOT, "paper_conf_cgo_qiaorht19_b200", "kcache")
+        old = [f for f in os.listdir(cache) if os.path.getmtime(os.path.join(cache, f)) < t0]
+        for f in old:
+            os.remove(os.path.join(cache, f))
+        print(f"pruned {len(old)} unused cubins")
     for e in errs:
         print("FAIL", e)
     sys.exit(1 if errs else 0)
