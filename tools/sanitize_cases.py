@@ -75,6 +75,26 @@ def main():
             for kind in ("unfused", "paper", "b200"):
                 run(spec, kind, seed=seed)
                 n += 1
+    if which in ("all", "peer"):
+        # the peer-halo kernels (kf_peer_signal / _pull / _wait) in ONE process: two
+        # row bands of a two-input image on this GPU, band 1 pulling band 0's last
+        # R rows of both inputs (any alignment: W = 130 is not a multiple of 4)
+        W, R = 130, 3
+        a = [torch.arange(20 * W, dtype=torch.float32, device="cuda").reshape(20, W) + 1000 * k for k in range(2)]
+        b = [torch.full((20 + R, W), -1.0, device="cuda") for _ in range(2)]
+        ctr_a = torch.zeros(8, dtype=torch.int32, device="cuda")
+        ctr_b = torch.zeros(8, dtype=torch.int32, device="cuda")
+        c = lambda t, i: t.data_ptr() + 4 * i   # noqa: E731
+        for step in range(3):
+            K.peer_signal([c(ctr_b, 0)], c(ctr_a, 6))
+            K.peer_pull([x.data_ptr() for x in b], [x.data_ptr() + (20 - R) * W * 4 for x in a], [R * W * 4] * 2,
+                        [c(ctr_b, 0)], [c(ctr_b, 2)], [c(ctr_a, 5)], c(ctr_b, 7), 1 << 20, copies=2)
+            K.peer_wait([c(ctr_a, 5)], [c(ctr_a, 6)], c(ctr_a, 7), 1 << 20)
+        torch.cuda.synchronize()
+        for k in range(2):
+            assert torch.equal(b[k][:R], a[k][20 - R:]), "peer pull"
+        assert int(ctr_a[7]) == 0 and int(ctr_b[7]) == 0 and int(ctr_b[2]) == 3
+        n += 3
     print(f"sanitize cases ok: {n} runs")
 
 
