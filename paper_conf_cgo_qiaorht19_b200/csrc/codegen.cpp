@@ -958,6 +958,7 @@ struct StreamGen {
     std::set<int> prp;     // external images fed by running row pointers from the prologue on (interior strips)
     bool qptr = false;     // steady-state loop: ring slots addressed from per-trip base pointers
     bool tma = false;      // this variant feeds the ring with TMA bulk row copies (option tma)
+    int peel_Q = 0;        // peeled iterations of the variant being emitted
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp},
@@ -978,15 +979,18 @@ struct StreamGen {
     // the prefetch of an external image) seen from loop-body copy j.  Unrolled:
     // slot = iteration mod P.  Rolled (one body copy, rings shifted by register
     // moves at the end of every iteration): slot = age (+D for external images).
+    // Rolled trips of T rows (si.T): body copy j of a trip sees its newest row
+    // at slot T-1-j, and the rings shift by T once per trip (peeled iterations
+    // are copy T-1 and shift by one), halving the moves for T = 2.
     int sl(int img, int off, int j) const
     {
         if (!si.rolled) return md(j + off, si.P);
-        return -off + (is_ext(img) && !si.sring ? si.D : 0);
+        return -off + (si.T - 1 - j) + (is_ext(img) && !si.sring ? si.D : 0);
     }
     int ring_len(int img) const
     {
         if (!si.rolled) return si.P;
-        return si.depth.at(img) + (is_ext(img) && !si.sring ? si.D : 0);
+        return si.depth.at(img) + si.T - 1 + (is_ext(img) && !si.sring ? si.D : 0);
     }
     std::string ring(int img, int s, int v) const
     {
@@ -1628,7 +1632,7 @@ struct StreamGen {
                 // this iteration's row is already in registers; wait for the next
                 // row and read it now, a whole iteration before its use
                 for (int img : b.ext) fetch(img, s_get, sl(img, 0, j), ind);
-                const bool wrap = !(u >= 0) && !(j + 1 < si.P && !si.rolled);
+                const bool wrap = !(u >= 0) && !(j + 1 < (si.rolled ? si.T : si.P));
                 const std::string s_nxt = u >= 0 ? std::to_string((u + 1) % DS)
                                                  : (!wrap ? "qb + " + std::to_string(j + 1) : "qnext");
                 const std::string p_nxt = u >= 0 ? std::to_string(((u + 1) / DS) & 1) : wrap ? "(ph ^ (qnext == 0))" : "ph";
@@ -1708,12 +1712,17 @@ struct StreamGen {
         }
         o << ind << "}\n";
         if (runptr) o << ind << "op += dW;\n";
-        if (si.rolled) {   // age every ring by one row
+        // age every ring: by one row after a peeled iteration (by T after the
+        // last one, which hands over to the first trip: there a row of age a sits
+        // at slot a + T - 1), by T rows after the last body copy of a rolled trip
+        const int shift = !si.rolled ? 0 : u >= 0 ? (u == peel_Q - 1 ? si.T : 1) : (j == si.T - 1 ? si.T : 0);
+        if (shift) {
             std::set<int> imgs(b.ext.begin(), b.ext.end());
             for (int k : b.kernels) imgs.insert(p->n_inputs + k);
             for (int img : imgs)
-                for (int a = ring_len(img) - 1; a >= 1; a--)
-                    for (int v = 0; v < NRi(img); v++) o << ind << ring(img, a, v) << " = " << ring(img, a - 1, v) << ";\n";
+                for (int a = ring_len(img) - 1; a >= shift; a--)
+                    for (int v = 0; v < NRi(img); v++)
+                        o << ind << ring(img, a, v) << " = " << ring(img, a - shift, v) << ";\n";
         }
         o << ind.substr(2) << "}\n";
     }
@@ -1856,14 +1865,21 @@ struct StreamGen {
                 if (p->ops[k].kind == LOCAL)
                     need = std::max(need, 2 * L - HY(p->n_inputs + k) + p->ops[k].ry());
         if (need > 0) {
-            const int Q = si.rolled ? need : (need + P - 1) / P * P;
-            for (int u = 0; u < Q; u++) iteration(u % P, u, std::to_string(u - u % P), "      ");
+            // rolled: a multiple of T, so that the ring slot qb + j of a trip stays below DS
+            const int Q = si.rolled ? (need + si.T - 1) / si.T * si.T : (need + P - 1) / P * P;
+            peel_Q = Q;
+            for (int u = 0; u < Q; u++) {
+                if (si.rolled)   // peeled rolled iterations are body copy T-1 (newest row at slot 0)
+                    iteration(si.T - 1, u, std::to_string(u - (si.T - 1)), "      ");
+                else
+                    iteration(u % P, u, std::to_string(u - u % P), "      ");
+            }
             u0 = Q;
             if (si.sring) o << "    qb = " << Q % si.DS << ";\n";
             if (tma) o << "    ph = " << ((Q / si.DS) & 1) << ";\n";
         }
         vedge = false;
-        const int step = si.rolled ? 1 : P;
+        const int step = si.rolled ? si.T : P;
         // steady state: running pointers for the next row to fetch into the ring and
         // the next output row (valid when the ring is deep enough that every row it
         // fetches after the prologue lies inside [base, rlast])
@@ -1881,11 +1897,12 @@ struct StreamGen {
             runptr = true;
         }
         if (si.rolled) {
+            const int T = si.T;
             o << "    #pragma unroll 1\n";
-            o << "    for (int u = " << u0 << "; u < nit; u++) {\n";
+            o << "    for (int u = " << u0 << "; u < nit; u += " << T << ") {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
-            if (si.lpf) o << "        const int qnext = qb + 1 == " << si.DS << " ? 0 : qb + 1;\n";
-            iteration(0, -1, "u", "        ");
+            if (si.lpf) o << "        const int qnext = qb + " << T << " == " << si.DS << " ? 0 : qb + " << T << ";\n";
+            for (int j = 0; j < T; j++) iteration(j, -1, "u", "        ");
         } else {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
@@ -2046,6 +2063,7 @@ const OptDef kOpts[] = {
     {"qptr", 1, 0, 1, false},           // per-trip ring slot base pointers
     {"heavy_first", 1, 0, 1, false},    // edge items first
     {"code_budget", 12000, 0, 1 << 30, false},   // unrolled vs rolled body
+    {"rtrip", 2, 1, 2, false},          // rows per trip of a rolled body (2: half the ring moves)
     {"rolled_edge_v", 1, 0, 1, false},  // rolled bodies keep the edge strips
     {"minctas", kMinCtasPerSm, 1, 32, false},    // __launch_bounds__ min CTAs per SM
     {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)
@@ -2249,6 +2267,14 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     // one rolled body copy
     const long long budget = opt(p, "code_budget");
     si.rolled = ops * si.P * 6 > budget;
+    // rows per rolled trip (option rtrip): 2 halves the ring-shift moves; the
+    // shared-memory ring then holds a multiple of T rows (slot qb + j < DS)
+    si.T = si.rolled && si.sring ? (int)opt(p, "rtrip") : 1;
+    if (si.T > 1) {
+        while (si.DS % si.T) si.DS += si.P;
+        if (si.DS % si.T) si.DS = si.DS * si.T;
+        si.ring_bytes = (int)b.ext.size() * si.DS * 128 * kV_;
+    }
     // rolled bodies keep the edge strips too (peeled remapped prologue, then
     // the rolled loop), unless option rolled_edge_v=0 leaves those rows to the
     // frame: for deep10 the frame's index-exchange tiles cost 12 % of the kernel

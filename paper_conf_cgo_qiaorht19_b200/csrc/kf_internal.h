@@ -146,6 +146,7 @@ struct StreamInfo {
     int D = 4;                    // prefetch distance (iterations)
     int live_regs = 0;            // estimate of ring registers
     bool rolled = false;          // one loop-body copy + ring shifts (big blocks)
+    int T = 1;                    // rows per rolled trip (body copies per rolled loop trip)
     bool sring = false;           // external rows fed by a cp.async shared-memory ring
     int DS = 0;                   // rows in that ring (multiple of P)
     bool lpf = false;             // ring rows read one iteration ahead (LDS latency off the critical path)
