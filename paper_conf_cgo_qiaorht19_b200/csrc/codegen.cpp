@@ -2063,7 +2063,8 @@ const OptDef kOpts[] = {
     {"qptr", 1, 0, 1, false},           // per-trip ring slot base pointers
     {"heavy_first", 1, 0, 1, false},    // edge items first
     {"code_budget", 12000, 0, 1 << 30, false},   // unrolled vs rolled body
-    {"rtrip", 2, 1, 2, false},          // rows per trip of a rolled body (2: half the ring moves)
+    {"rtrip", 1, 1, 2, false},          // rows per trip of a rolled body (2: half the ring moves, but
+                                        // twice the loop code: measured slower, instruction fetch stalls)
     {"rolled_edge_v", 1, 0, 1, false},  // rolled bodies keep the edge strips
     {"minctas", kMinCtasPerSm, 1, 32, false},    // __launch_bounds__ min CTAs per SM
     {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)

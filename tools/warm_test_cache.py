@@ -52,8 +52,8 @@ def jobs():
             out.append((P.WORKLOADS[wl](2048, 2048), kind, None, False))
     same = [{"qptr": 0}, {"lds_pf": 0}, {"const_w": 0}, {"heavy_first": 0}, {"pro_rp": 0}, {"smem_rows": 6},
             {"sring": 0}, {"minctas": 8}, {"code_budget": 1000}, {"swring": 0}, {"tma": 1},
-            {"tma": 1, "lds_pf": 0}, {"tma": 1, "code_budget": 1000}, {"tma": 1, "smem_rows": 6}, {"rtrip": 1},
-            {"rtrip": 1, "code_budget": 1000}, {"code_budget": 1000, "lds_pf": 0}]
+            {"tma": 1, "lds_pf": 0}, {"tma": 1, "code_budget": 1000}, {"tma": 1, "smem_rows": 6}, {"rtrip": 2},
+            {"rtrip": 2, "code_budget": 1000}, {"code_budget": 1000, "lds_pf": 0}]
     exp = [{"v8": 1}, {"persist": 1}, {"nlong": 3}]
     for wl in ["harris", "unsharp", "shitomasi"]:
         for o in ({"pairs": 0}, {"defer": 0}):
@@ -63,8 +63,8 @@ def jobs():
         out.append((spec, "b200", {"tma": 1}, False))
     out.append((P.copy(4096, 4096), "b200", {"tma": 1}, False))
     out.append((P.copy(4096, 4096), "b200", None, False))
-    out.append((P.config("C4")[0], "b200", {"rtrip": 1}, False))
-    out.append((P.enhance(2048, 2048), "b200", {"rtrip": 1}, False))
+    out.append((P.config("C4")[0], "b200", {"rtrip": 2}, False))
+    out.append((P.enhance(2048, 2048), "b200", {"rtrip": 2}, False))
     for wl in ["harris", "deep10", "unsharp"]:
         for o in same:
             out.append((P.WORKLOADS[wl](200, 150), "b200", o, False))
