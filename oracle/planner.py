@@ -52,10 +52,16 @@ class Model:
     tile_w: int = 32
     tile_h: int = 32
     eq3_mode: int = 0       # 0: IS*tg/ts as printed; 1: IS*(tg-ts)  (O1-a)
+    bw_bytes_clk: float = 0.0      # phi_mode 2 (ROOFLINE, R-20) only
+    issue_lanes_clk: float = 0.0
 
 
 PAPER_PROFILE = Model()
 B200_PROFILE = Model(c_mshared=5.0, phi_mode=1)
+# the B200 issue-rate extension (R-20; constants of kfuse.h
+# kf_model_params_b200_roofline, restated)
+B200_ROOF_PROFILE = Model(c_alu=1.0, c_sfu=40.0, c_mshared=5.0, phi_mode=2, tile_w=120, tile_h=32,
+                          bw_bytes_clk=22.45, issue_lanes_clk=115.0)
 
 
 @dataclass
@@ -70,6 +76,7 @@ class Graph:
     outputs: set
     bpp: int
     cost: list                   # (n_alu, n_sfu)
+    u8: bool = False             # u8x4 pipeline
     edges: list = field(default_factory=list)   # (ks, kd) unique, consumer-major order
     consumers: list = field(default_factory=list)
     producers: list = field(default_factory=list)
@@ -97,7 +104,7 @@ def graph(spec: dict) -> Graph:
               rx=[len(o["mask"][0]) // 2 if o["kind"] == "local" else 0 for o in ops],
               ry=[len(o["mask"]) // 2 if o["kind"] == "local" else 0 for o in ops],
               mode=[o.get("mode") for o in ops], outputs=set(spec["outputs"]),
-              bpp=4, cost=[kernel_costs(o) for o in ops])
+              bpp=4, cost=[kernel_costs(o) for o in ops], u8=spec["dtype"] == "u8x4")
     g.consumers = [[] for _ in ops]
     g.producers = [[] for _ in ops]
     for kd, o in enumerate(ops):
@@ -184,8 +191,34 @@ class EdgeInfo:
     weight: tuple     # (q, eps)
 
 
+def roofline_time(g: Graph, kernels: list, m: Model) -> float:
+    """ROOFLINE reading R-20: SM-cycles per pixel of `kernels` (one kernel, or a
+    producer followed by its consumer) fused into one kernel = max(DRAM time,
+    issue time).  DRAM: 4 B per distinct image read from outside plus the one
+    output; issue: Eq. 6's cost as issue slots per pixel (x2 for u8x4's two SWAR
+    channel pairs), the producer recomputed on the consumer's staged halo."""
+    inside = {g.n_inputs + k for k in kernels}
+    read = sorted({i for k in kernels for i in g.inputs[k] if i not in inside})
+    per_ch = 2.0 if g.bpp == 4 and g.u8 else 1.0
+    slots = []
+    for pos, k in enumerate(kernels):
+        n_alu, n_sfu = g.cost[k]
+        c = (m.c_alu * n_alu + m.c_sfu * n_sfu) * per_ch
+        if pos == 0 and len(kernels) == 2 and g.kind[kernels[1]] == "local":
+            kd = kernels[1]
+            c *= (m.tile_w + 2 * g.rx[kd]) * (m.tile_h + 2 * g.ry[kd]) / (m.tile_w * m.tile_h)
+        slots.append(c)
+    dram = g.bpp * (len(read) + 1) / m.bw_bytes_clk
+    issue = sum(slots) / m.issue_lanes_clk
+    return dram if dram > issue else issue
+
+
 def benefit(g: Graph, ks: int, kd: int, m: Model) -> tuple[str, float]:
     """w for edge (ks, kd) by scenario, Eqs. 3-11, plus gamma (Eq. 12)."""
+    if m.phi_mode == 2:                          # ROOFLINE reading R-20
+        sc = "point" if g.kind[kd] == "point" else ("p2l" if g.kind[ks] == "point" else "l2l")
+        w = roofline_time(g, [ks], m) + roofline_time(g, [kd], m) - roofline_time(g, [ks, kd], m)
+        return sc, w + m.gamma
     IS = 1.0                                     # reading O1-c (PAPER.md:710-711)
     n_alu, n_sfu = g.cost[ks]
     costop = m.c_alu * n_alu + m.c_sfu * n_sfu   # Eq. 6

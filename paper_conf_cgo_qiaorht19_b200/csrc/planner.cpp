@@ -114,6 +114,29 @@ static bool context_legal(const kf_pipeline *p, const std::set<int> &P, const kf
     return dependence_legal(p, P) && resource_legal(p, P, m) && header_legal(p, P);
 }
 
+// ROOFLINE reading (phi_mode 2, R-20): SM-cycles per pixel of the
+// kernel set {ks} or {ks, kd} run as one kernel -- the larger of its DRAM
+// time (bpp bytes per distinct external image and per output) and its issue
+// time (Eq. 6 costs as issue slots, the producer recomputed on the staged halo).
+static double roof_time(const kf_pipeline *p, int ks, int kd, const kf_model_params &m)
+{
+    const double ch = p->dtype == KF_U8X4 ? 2.0 : 1.0;
+    auto issue = [&](int k) { const Op &o = p->ops[k]; return (m.c_alu * o.n_alu + m.c_sfu * o.n_sfu) * ch; };
+    std::set<int> ext(p->ops[ks].inputs.begin(), p->ops[ks].inputs.end());
+    double slots = issue(ks);
+    if (kd >= 0) {
+        const Op &d = p->ops[kd];
+        for (int i : d.inputs)
+            if (i != p->n_inputs + ks) ext.insert(i);
+        const double r = d.kind == LOCAL ? (double)((m.tile_w + 2 * d.rx()) * (m.tile_h + 2 * d.ry())) /
+                                                   (double)(m.tile_w * m.tile_h)
+                                         : 1.0;
+        slots = issue(ks) * r + issue(kd);
+    }
+    const double mem = 4.0 * (double)(ext.size() + 1) / m.bw_bytes_clk;
+    return std::max(mem, slots / m.issue_lanes_clk);
+}
+
 // Benefit of one edge, Eqs. 3-11 plus gamma (Eq. 12 before clamping).
 static EdgeInfo benefit(const kf_pipeline *p, int ks, int kd, const kf_model_params &m)
 {
@@ -124,6 +147,11 @@ static EdgeInfo benefit(const kf_pipeline *p, int ks, int kd, const kf_model_par
     EdgeInfo e{};
     e.ks = ks;
     e.kd = kd;
+    if (m.phi_mode == 2) {                                    // ROOFLINE (R-20)
+        e.scenario = d.kind == POINT ? 0 : s.kind == POINT ? 1 : 2;
+        e.w = roof_time(p, ks, -1, m) + roof_time(p, kd, -1, m) - roof_time(p, ks, kd, m) + m.gamma;
+        return e;
+    }
     if (d.kind == POINT) {                                    // point-based, Eqs. 4-5
         e.scenario = 0;
         e.w = IS * m.tg + m.gamma;

@@ -39,7 +39,8 @@ class KfCost(C.Structure):
 class ModelParams(C.Structure):
     _fields_ = [("tg", C.c_double), ("ts", C.c_double), ("c_alu", C.c_double), ("c_sfu", C.c_double),
                 ("gamma", C.c_double), ("c_mshared", C.c_double), ("phi_mode", C.c_int32),
-                ("tile_w", C.c_int32), ("tile_h", C.c_int32), ("eq3_mode", C.c_int32)]
+                ("tile_w", C.c_int32), ("tile_h", C.c_int32), ("eq3_mode", C.c_int32),
+                ("bw_bytes_clk", C.c_double), ("issue_lanes_clk", C.c_double)]
 
 
 class KfError(RuntimeError):
@@ -54,6 +55,7 @@ _I32P = C.POINTER(C.c_int32)
 _SIGS = {
     "kf_model_params_paper": (None, [C.POINTER(ModelParams)]),
     "kf_model_params_b200": (None, [C.POINTER(ModelParams)]),
+    "kf_model_params_b200_roofline": (None, [C.POINTER(ModelParams)]),
     "kf_pipeline_create": (C.c_int, [C.c_int32, C.c_int32, C.c_int, C.POINTER(_P)]),
     "kf_pipeline_destroy": (None, [_P]),
     "kf_add_input": (C.c_int, [_P, _I32P]),
@@ -116,7 +118,8 @@ def _check(st: int) -> None:
 
 def model_params(profile: str = "paper", **over) -> ModelParams:
     m = ModelParams()
-    (lib.kf_model_params_b200 if profile == "b200" else lib.kf_model_params_paper)(C.byref(m))
+    {"b200": lib.kf_model_params_b200, "b200roof": lib.kf_model_params_b200_roofline}.get(
+        profile, lib.kf_model_params_paper)(C.byref(m))
     for k, v in over.items():
         setattr(m, k, v)
     return m

@@ -27,7 +27,7 @@ def test_exports_every_declared_symbol():
 
 
 def _ref_model(profile):
-    return PL.PAPER_PROFILE if profile == "paper" else PL.B200_PROFILE
+    return {"paper": PL.PAPER_PROFILE, "b200": PL.B200_PROFILE, "b200roof": PL.B200_ROOF_PROFILE}[profile]
 
 
 def _compare(spec, profile):
@@ -44,10 +44,19 @@ def _compare(spec, profile):
     return plan
 
 
-@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10"])
-@pytest.mark.parametrize("profile", ["paper", "b200"])
+@pytest.mark.parametrize("wl", ["harris", "shitomasi", "unsharp", "sobel", "enhance", "deep10", "two_input"])
+@pytest.mark.parametrize("profile", ["paper", "b200", "b200roof"])
 def test_planner_matches_reference_on_workloads(wl, profile):
     _compare(P.WORKLOADS[wl](64, 64), profile)
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_roofline_planner_matches_reference_on_random_dags(seed):
+    """The ROOFLINE profile (R-20): edge weights, cuts and partition equal the
+    independent Python planner's on random DAGs of both dtypes."""
+    rng = random.Random(61000 + seed)
+    spec = P.random_pipeline(rng, 40, 30, rng.choice(["f32", "u8x4"]), rng.randint(2, 8))
+    _compare(spec, "b200roof")
 
 
 def test_harris_plan_pins_through_the_abi():

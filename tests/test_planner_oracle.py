@@ -306,3 +306,71 @@ def test_basic_fusion_is_legal_cover_below_optimum(seed):
         assert PL.basic_legal(g, set(b), m, info)
         beta = PL._add(beta, PL.block_weight(set(b), info))
     assert beta <= PL.brute_force(s, m)[0]
+
+
+# ------------------------------------------------ ROOFLINE extension (R-20)
+
+def _chain(prog1, prog2, local2=None, dtype="f32"):
+    p = P.Pipeline("chain", 64, 64, dtype)
+    i = p.input()
+    a = p.point("a", [i], prog1)
+    b = p.local("b", a, local2, "clamp") if local2 else p.point("b", [a], prog2)
+    p.output(b)
+    return p.spec()
+
+
+def test_roofline_memory_bound_pair_saves_the_intermediate_image():
+    """Two cheap point kernels: each moves 8 B/px unfused, the fused pair 8 B/px,
+    so the benefit is exactly the intermediate's write + read, 2 * 4 B / bw."""
+    m = PL.B200_ROOF_PROFILE
+    s = _chain([P.L(0), P.C(1.0), P.ADD], [P.L(0), P.C(2.0), P.MUL])
+    info = PL.edge_weights(PL.graph(s), m)
+    assert info[(0, 1)].w == pytest.approx(8.0 / m.bw_bytes_clk, rel=1e-12)
+    assert info[(0, 1)].profitable
+
+
+def test_roofline_issue_bound_pair_gains_nothing():
+    """Two POW-heavy point kernels, each issue-bound alone: fusing saves DRAM time
+    that was hidden anyway, so w = 0 -- unprofitable, an eps edge (Eq. 12, R-3)."""
+    m = PL.B200_ROOF_PROFILE
+    heavy = [P.L(0), P.C(0.5), P.POW, P.C(0.7), P.POW, P.C(0.9), P.POW]
+    s = _chain(heavy, heavy)
+    g = PL.graph(s)
+    assert PL.roofline_time(g, [0], m) > 4 * 2 / m.bw_bytes_clk      # issue-bound alone
+    info = PL.edge_weights(g, m)
+    assert info[(0, 1)].w == pytest.approx(0.0, abs=1e-12) and not info[(0, 1)].profitable
+    assert info[(0, 1)].weight == (0, 1)
+
+
+def test_roofline_issue_bound_producer_recompute_costs_its_halo():
+    """An issue-bound producer feeding a 3x3 local kernel is recomputed on the
+    staged halo: the pair costs I(producer) * (tw+2)(th+2)/(tw th) + I(consumer)
+    issue slots, which outweighs the consumer's hidden DRAM time when the
+    producer is heavy enough -> w < 0, unprofitable."""
+    m = PL.B200_ROOF_PROFILE
+    heavy = [P.L(0)] + [t for _ in range(15) for t in (P.C(0.99), P.POW)]   # 15 POW: ~600 issue slots / px
+    s = _chain(heavy, None, local2=[[1, 1, 1]] * 3)
+    g = PL.graph(s)
+    n_alu, n_sfu = g.cost[0]
+    i0 = m.c_alu * n_alu + m.c_sfu * n_sfu
+    fac = (m.tile_w + 2) * (m.tile_h + 2) / (m.tile_w * m.tile_h)
+    t0, t1 = PL.roofline_time(g, [0], m), PL.roofline_time(g, [1], m)
+    w = PL.edge_weights(g, m)[(0, 1)].w
+    # the consumer alone is memory-bound, the fused pair issue-bound
+    assert t1 == pytest.approx(8.0 / m.bw_bytes_clk)
+    assert w == pytest.approx(t0 + t1 - (i0 * fac + g.cost[1][0] * m.c_alu) / m.issue_lanes_clk, rel=1e-12)
+    assert w < 0 and not PL.edge_weights(g, m)[(0, 1)].profitable
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_roofline_plan_bounded_by_bruteforce(seed):
+    """Alg. 1 under the ROOFLINE weights: legal cover, beta <= the exhaustive optimum."""
+    rng = random.Random(5100 + seed)
+    s = P.random_pipeline(rng, 16, 16, rng.choice(["f32", "u8x4"]), rng.randint(2, 7))
+    m = PL.B200_ROOF_PROFILE
+    pl = PL.get_legal_partitions(s, m)
+    g = PL.graph(s)
+    assert sorted(k for b in pl.blocks for k in b) == list(range(g.n))
+    for b in pl.blocks:
+        assert PL.is_legal(g, set(b), m, pl.info)
+    assert pl.beta <= PL.brute_force(s, m)[0]

@@ -10,13 +10,16 @@
    chunk by a 32-row strip -- and cMshared = 5.
 2. For every paper application (Harris, ShiTomasi, Unsharp, Sobel, Enhance, and
    the deep10 C4 body) at the paper's 2048x2048 size: the named plans (unfused,
-   basic [12], Alg. 1 under the paper / B200 / b200cal profiles, the exact
-   optimum under b200cal) plus random executable partitions (random merges along
+   basic [12], Alg. 1 under the paper / B200 / b200cal / b200roof profiles, the
+   exact optimum under b200cal and b200roof) plus random executable partitions (random merges along
    edges accepted by kf_plan_from_blocks).  Each plan's objective beta (Eq. 1:
    the sum of the b200cal weights of the edges inside blocks; eps edges count 0
    with their number reported) is set against its measured time (CUDA-graph
    replay, 4 rotating buffer sets).  Spearman's rank correlation between beta
-   and time says whether the calibrated model ranks plans the way B200 does.
+   and time says whether the calibrated model ranks plans the way B200 does --
+   for the b200cal weights (the paper's Eqs. 3-12 with measured latencies) and
+   for the ROOFLINE weights (R-20: per-pair max(DRAM time, issue
+   time), the issue-rate extension for compute-bound blocks).
 3. Table I shape: speedups of basic and optimized fusion over unfused, and of
    optimized over basic, per application.
 
@@ -120,6 +123,10 @@ def random_partitions(spec, rng, n_samples, tries=400) -> list:
     return out
 
 
+def t_of(rows, name):
+    return next(r["us"] for r in rows if r["plan"] == name)
+
+
 def spearman(x, y) -> float:
     def ranks(v):
         order = sorted(range(len(v)), key=lambda i: v[i])
@@ -142,12 +149,43 @@ def spearman(x, y) -> float:
     return cov / (vx * vy) if vx > 0 and vy > 0 else float("nan")
 
 
+def _compile_labels(job):
+    app, size, lab = job
+    spec = P.WORKLOADS[app](size, size)
+    K.Pipeline.from_spec(spec).plan_from_blocks(lab).compile()
+
+
+def compile_only(size: int, samples: int) -> None:
+    """Warms the in-tree cubin cache with every plan main() will time (no GPU)."""
+    from multiprocessing import Pool
+    rng = random.Random(2019)
+    jobs = []
+    for app in APPS:
+        spec = P.WORKLOADS[app](size, size)
+        p = K.Pipeline.from_spec(spec)
+        for plan in (p.plan_unfused(), p.plan_basic("paper"), p.plan_fusion("paper"), p.plan_fusion("b200"),
+                     p.plan_fusion("b200roof"), p.plan_exact("b200roof")):
+            lab = [0] * len(spec["ops"])
+            for bi, ks in enumerate(plan.blocks):
+                for k in ks:
+                    lab[k] = bi
+            jobs.append((app, size, lab))
+        jobs += [(app, size, lab) for lab in random_partitions(spec, rng, samples)]
+    with Pool(os.cpu_count()) as pool:
+        pool.map(_compile_labels, jobs, chunksize=1)
+    print(f"compiled {len(jobs)} plans")
+
+
 def main():
     ap = argparse.ArgumentParser()
+    ap.add_argument("--compile-only", action="store_true")
     ap.add_argument("--size", type=int, default=2048)
-    ap.add_argument("--samples", type=int, default=14)
+    ap.add_argument("--samples", type=int, default=24)
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "calibration.json"))
     a = ap.parse_args()
+    if a.compile_only:
+        compile_only(a.size, a.samples)
+        return
     consts = measure_consts()
     mcal = cal_params(consts)
     print(json.dumps({"consts": consts}), flush=True)
@@ -162,12 +200,16 @@ def main():
         oshape = (H, W) if spec["dtype"] == "f32" else (H, W, 4)
         ins = [torch.from_numpy(host).cuda() for _ in range(4)]
         outs = [torch.empty(oshape, dtype=tdt, device="cuda") for _ in range(4)]
-        ref = K.Pipeline.from_spec(spec).plan_fusion(mcal)
-        weights = {}
-        for k, o in enumerate(spec["ops"]):
-            for img in o["inputs"]:
-                if img >= spec["n_inputs"]:
-                    weights[(img - spec["n_inputs"], k)] = ref.edge(img - spec["n_inputs"], k)
+        def edge_table(prof):
+            ref = K.Pipeline.from_spec(spec).plan_fusion(prof)
+            wt = {}
+            for k, o in enumerate(spec["ops"]):
+                for img in o["inputs"]:
+                    if img >= spec["n_inputs"]:
+                        wt[(img - spec["n_inputs"], k)] = ref.edge(img - spec["n_inputs"], k)
+            return wt
+        weights = edge_table(mcal)
+        weights_roof = edge_table(K.model_params("b200roof"))
         named = {
             "unfused": lambda p: p.plan_unfused(),
             "basic": lambda p: p.plan_basic("paper"),
@@ -175,6 +217,8 @@ def main():
             "alg1_b200": lambda p: p.plan_fusion("b200"),
             "alg1_b200cal": lambda p: p.plan_fusion(mcal),
             "exact_b200cal": lambda p: p.plan_exact(mcal),
+            "alg1_b200roof": lambda p: p.plan_fusion("b200roof"),
+            "exact_b200roof": lambda p: p.plan_exact("b200roof"),
         }
         rows = []
         done = set()
@@ -182,9 +226,10 @@ def main():
             plan = mk(K.Pipeline.from_spec(spec))
             key = tuple(map(tuple, plan.blocks))
             b, ne = beta(plan.blocks, weights)
+            br, _ = beta(plan.blocks, weights_roof)
             us = time_plan(plan, ins, outs)
             rows.append({"plan": name, "blocks": plan.blocks, "beta": round(b, 2), "eps": ne,
-                         "launches": plan.num_launches, "us": round(us, 2)})
+                         "beta_roof": round(br, 5), "launches": plan.num_launches, "us": round(us, 2)})
             done.add(key)
         for lab in random_partitions(spec, rng, a.samples):
             plan = K.Pipeline.from_spec(spec).plan_from_blocks(lab)
@@ -193,14 +238,18 @@ def main():
                 continue
             done.add(key)
             b, ne = beta(plan.blocks, weights)
+            br, _ = beta(plan.blocks, weights_roof)
             us = time_plan(plan, ins, outs)
             rows.append({"plan": "random", "blocks": plan.blocks, "beta": round(b, 2), "eps": ne,
-                         "launches": plan.num_launches, "us": round(us, 2)})
+                         "beta_roof": round(br, 5), "launches": plan.num_launches, "us": round(us, 2)})
         t = {r["plan"]: r["us"] for r in rows if r["plan"] != "random"}
         rho = spearman([r["beta"] for r in rows], [r["us"] for r in rows])
+        rho_roof = spearman([r["beta_roof"] for r in rows], [r["us"] for r in rows])
         best = min(rows, key=lambda r: r["us"])
         d = {"workload": f"{app} {W}x{H} {spec['dtype']}", "plans": rows,
              "spearman_beta_vs_time": round(rho, 3),
+             "spearman_beta_roof_vs_time": round(rho_roof, 3),
+             "alg1_b200roof_us": t_of(rows, "alg1_b200roof"), "alg1_b200_us": t_of(rows, "alg1_b200"),
              "fastest": best["plan"], "fastest_blocks": best["blocks"],
              "table1": {"basic_over_unfused": round(t["unfused"] / t["basic"], 3),
                         "optimized_paper_over_unfused": round(t["unfused"] / t["alg1_paper"], 3),
