@@ -120,22 +120,25 @@ typedef struct { int32_t n_alu; int32_t n_sfu; } kf_cost;
  *                     (tile_w+2rx)(tile_h+2ry)/(tile_w*tile_h)  (R-4)
  *   eq3_mode      0 = delta_Mshared = IS*tg/ts as printed (Eq. 3); 1 = IS*(tg-ts)
  *   phi_mode 2 = ROOFLINE (R-20, the B200 issue-rate extension): a
- *     kernel set S fused into one kernel takes
- *       T(S) = max( bpp * (|external inputs| + 1) / bw_bytes_clk,
- *                   sum_k costop(k) * ch * r_S(k) / issue_lanes_clk )
- *     SM-cycles per pixel (costop of Eq. 6 read as issue slots per pixel, ch = 2
- *     for U8X4 -- two SWAR channel pairs -- else 1, r_S(k) the staged halo
- *     recompute factor of the producer inside S, as in STAGED), and an edge's
- *     benefit is w = T({ks}) + T({kd}) - T({ks, kd}) + gamma: memory savings
- *     count only while the pair stays memory-bound, recompute only when it is
- *     issue-bound.  tg/ts are unused.
+ *     kernel set S fused into one kernel takes, in SM-cycles per pixel,
+ *       M(S) = bpp * (|external input images| + 1) / bw_bytes_clk     (DRAM)
+ *       C(S) = sum_k slots(k) * ch * r_S(k) / issue_lanes_clk           (issue)
+ *       T(S) = max(M, C) + overlap * min(M, C)
+ *     (overlap 0: a perfect roofline, 1: no overlap, M + C).  slots(k) = issue
+ *     slots per pixel of kernel k: every program opcode except LOAD/CONST
+ *     counts 1, except POW 80, LOG 30, EXP 25, SQRT 2, DIV 15 (their SASS
+ *     expansion on sm_100a), plus one per non-zero mask tap of a local kernel;
+ *     ch = 2 for U8X4 (two SWAR channel pairs) else 1; r_S(k) is the staged
+ *     halo recompute factor of the producer inside S, as in STAGED.  An edge's
+ *     benefit is w = T({ks}) + T({kd}) - T({ks, kd}) + gamma.  tg, ts, c_alu,
+ *     c_sfu and kf_cost are unused in this mode.
  * kf_model_params_paper(): tg=400 ts=4 c_alu=4 c_sfu=16 gamma=0 c_mshared=2
  *   phi PAPER, 32x32.  kf_model_params_b200(): same but
  *   c_mshared=5, phi STAGED. */
 typedef struct {
     double tg, ts, c_alu, c_sfu, gamma, c_mshared;
     int32_t phi_mode, tile_w, tile_h, eq3_mode;
-    double bw_bytes_clk, issue_lanes_clk;   /* phi_mode 2 only (see below) */
+    double bw_bytes_clk, issue_lanes_clk, overlap;   /* phi_mode 2 only (see below) */
 } kf_model_params;
 
 typedef struct kf_pipeline kf_pipeline;
@@ -143,10 +146,10 @@ typedef struct kf_plan kf_plan;
 
 void kf_model_params_paper(kf_model_params *p);
 void kf_model_params_b200(kf_model_params *p);
-/* kf_model_params_b200_roofline(): phi_mode 2 with B200 constants: c_alu = 1
- * issue slot per ALU op, c_sfu = 40 (average SASS expansion of an accurate
- * log/exp/pow), bw_bytes_clk = 22.45 (6528 GB/s measured copy / 148 SMs /
- * 1965 MHz), issue_lanes_clk = 115 (measured FFMA rate 3.6 warp-instr/clk/SM),
+/* kf_model_params_b200_roofline(): phi_mode 2 with B200 constants:
+ * bw_bytes_clk = 22.45 (6528 GB/s measured copy / 148 SMs / 1965 MHz),
+ * issue_lanes_clk = 115 (measured FFMA rate 3.6 warp-instr/clk/SM), overlap 1
+ * (fitted: best rank correlation with measured plan times, R-20),
  * tile 120x32 (the streaming chunk), c_mshared = 5, gamma = 0. */
 void kf_model_params_b200_roofline(kf_model_params *p);
 

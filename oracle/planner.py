@@ -54,14 +54,17 @@ class Model:
     eq3_mode: int = 0       # 0: IS*tg/ts as printed; 1: IS*(tg-ts)  (O1-a)
     bw_bytes_clk: float = 0.0      # phi_mode 2 (ROOFLINE, R-20) only
     issue_lanes_clk: float = 0.0
+    overlap: float = 0.0
 
 
 PAPER_PROFILE = Model()
 B200_PROFILE = Model(c_mshared=5.0, phi_mode=1)
 # the B200 issue-rate extension (R-20; constants of kfuse.h
 # kf_model_params_b200_roofline, restated)
-B200_ROOF_PROFILE = Model(c_alu=1.0, c_sfu=40.0, c_mshared=5.0, phi_mode=2, tile_w=120, tile_h=32,
-                          bw_bytes_clk=22.45, issue_lanes_clk=115.0)
+B200_ROOF_PROFILE = Model(c_mshared=5.0, phi_mode=2, tile_w=120, tile_h=32,
+                          bw_bytes_clk=22.45, issue_lanes_clk=115.0, overlap=1.0)
+# issue slots per pixel of an op-IR opcode (restated from include/kfuse.h, phi_mode 2)
+ISSUE_SLOTS = {"LOAD": 0, "CONST": 0, "POW": 80, "LOG": 30, "EXP": 25, "SQRT": 2, "DIV": 15}
 
 
 @dataclass
@@ -77,6 +80,8 @@ class Graph:
     bpp: int
     cost: list                   # (n_alu, n_sfu)
     u8: bool = False             # u8x4 pipeline
+    progs: list = field(default_factory=list)   # point body / local post program per kernel
+    taps: list = field(default_factory=list)    # non-zero mask entries per kernel (0 for point)
     edges: list = field(default_factory=list)   # (ks, kd) unique, consumer-major order
     consumers: list = field(default_factory=list)
     producers: list = field(default_factory=list)
@@ -104,7 +109,9 @@ def graph(spec: dict) -> Graph:
               rx=[len(o["mask"][0]) // 2 if o["kind"] == "local" else 0 for o in ops],
               ry=[len(o["mask"]) // 2 if o["kind"] == "local" else 0 for o in ops],
               mode=[o.get("mode") for o in ops], outputs=set(spec["outputs"]),
-              bpp=4, cost=[kernel_costs(o) for o in ops], u8=spec["dtype"] == "u8x4")
+              bpp=4, cost=[kernel_costs(o) for o in ops], u8=spec["dtype"] == "u8x4",
+              progs=[list(o["prog"] if o["kind"] == "point" else o["post"]) for o in ops],
+              taps=[sum(1 for r in o["mask"] for v in r if v != 0.0) if o["kind"] == "local" else 0 for o in ops])
     g.consumers = [[] for _ in ops]
     g.producers = [[] for _ in ops]
     for kd, o in enumerate(ops):
@@ -193,24 +200,25 @@ class EdgeInfo:
 
 def roofline_time(g: Graph, kernels: list, m: Model) -> float:
     """ROOFLINE reading R-20: SM-cycles per pixel of `kernels` (one kernel, or a
-    producer followed by its consumer) fused into one kernel = max(DRAM time,
-    issue time).  DRAM: 4 B per distinct image read from outside plus the one
-    output; issue: Eq. 6's cost as issue slots per pixel (x2 for u8x4's two SWAR
-    channel pairs), the producer recomputed on the consumer's staged halo."""
+    producer followed by its consumer) fused into one kernel =
+    max(M, C) + overlap * min(M, C).  M (DRAM): 4 B per distinct image read
+    from outside plus the one output; C (issue): the kernels' issue slots per
+    pixel (ISSUE_SLOTS per opcode, one per non-zero mask tap; x2 for u8x4's two
+    SWAR channel pairs), the producer recomputed on the consumer's staged halo."""
     inside = {g.n_inputs + k for k in kernels}
     read = sorted({i for k in kernels for i in g.inputs[k] if i not in inside})
     per_ch = 2.0 if g.bpp == 4 and g.u8 else 1.0
     slots = []
     for pos, k in enumerate(kernels):
-        n_alu, n_sfu = g.cost[k]
-        c = (m.c_alu * n_alu + m.c_sfu * n_sfu) * per_ch
+        c = float(sum(ISSUE_SLOTS.get(t[0], 1) for t in g.progs[k]) + g.taps[k]) * per_ch
         if pos == 0 and len(kernels) == 2 and g.kind[kernels[1]] == "local":
             kd = kernels[1]
             c *= (m.tile_w + 2 * g.rx[kd]) * (m.tile_h + 2 * g.ry[kd]) / (m.tile_w * m.tile_h)
         slots.append(c)
     dram = g.bpp * (len(read) + 1) / m.bw_bytes_clk
     issue = sum(slots) / m.issue_lanes_clk
-    return dram if dram > issue else issue
+    hi, lo = (dram, issue) if dram > issue else (issue, dram)
+    return hi + m.overlap * lo
 
 
 def benefit(g: Graph, ks: int, kd: int, m: Model) -> tuple[str, float]:

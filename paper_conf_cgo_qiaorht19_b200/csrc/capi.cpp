@@ -73,6 +73,7 @@ void kf_model_params_paper(kf_model_params *m)
     m->eq3_mode = 0;
     m->bw_bytes_clk = 0.0;
     m->issue_lanes_clk = 0.0;
+    m->overlap = 0.0;
 }
 
 void kf_model_params_b200(kf_model_params *m)
@@ -89,12 +90,11 @@ void kf_model_params_b200_roofline(kf_model_params *m)
     if (!m) return;
     m->phi_mode = 2;          // DESIGN.md R-20
     m->c_mshared = 5.0;
-    m->c_alu = 1.0;           // issue slots per ALU op
-    m->c_sfu = 40.0;          // SASS expansion of an accurate logf/expf/powf (tools/ubench, codegen prog_size)
     m->tile_w = 120;          // streaming column chunk (32 - 2 halo lanes) x 4 pixels ...
     m->tile_h = 32;           // ... by a strip of rows
     m->bw_bytes_clk = 22.45;  // 6528.4 GB/s / (148 SMs x 1.965 GHz)
     m->issue_lanes_clk = 115.0;   // 3.6 FFMA warp-instr / clk / SM (profiles/r01_fp_int_issue_rates.txt)
+    m->overlap = 1.0;             // fitted (profiles/r02_calibration.md)
 }
 
 kf_status kf_pipeline_create(int32_t width, int32_t height, kf_dtype dtype, kf_pipeline **out)

@@ -2136,16 +2136,7 @@ long long get_option(const kf_pipeline *p, const char *name)
 static int prog_size(const Op &op)
 {
     int n = 0;
-    for (const Instr &in : op.prog) {
-        switch (in.op) {
-        case KF_OP_POW: n += 80; break;
-        case KF_OP_LOG: n += 30; break;
-        case KF_OP_EXP: n += 25; break;
-        case KF_OP_SQRT: n += 2; break;   // MUFU.SQRT (kf_sqrt)
-        case KF_OP_DIV: n += 15; break;
-        default: n += 1;
-        }
-    }
+    for (const Instr &in : op.prog) n += std::max(1, op_issue_slots(in.op));   // LOAD/CONST count 1 here
     return n;
 }
 

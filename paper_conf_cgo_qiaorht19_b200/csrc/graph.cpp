@@ -58,6 +58,23 @@ void validate_program(const kf_pipeline *p, const std::vector<Instr> &prog, int 
 }
 
 // nALU / nSFU default to an opcode count (R-3).
+// Issue slots per pixel of one op-IR instruction on sm_100a: 1, except the
+// accurate transcendental / division sequences (SASS expansion, fitted to
+// cuobjdump counts).  Shared by the code-size estimate (codegen.cpp) and the
+// ROOFLINE benefit (planner.cpp, R-20).
+int op_issue_slots(int opcode)
+{
+    switch (opcode) {
+    case KF_OP_LOAD: case KF_OP_CONST: return 0;
+    case KF_OP_POW: return 80;
+    case KF_OP_LOG: return 30;
+    case KF_OP_EXP: return 25;
+    case KF_OP_SQRT: return 2;   // MUFU.SQRT (kf_sqrt)
+    case KF_OP_DIV: return 15;
+    default: return 1;
+    }
+}
+
 void default_cost(const kf_pipeline *, Op &op)
 {
     int alu = 0, sfu = 0;

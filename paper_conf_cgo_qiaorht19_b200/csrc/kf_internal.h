@@ -110,6 +110,7 @@ namespace kf {
 // graph.cpp
 void validate_program(const kf_pipeline *p, const std::vector<Instr> &prog, int n_loads, bool has_lut);
 void default_cost(const kf_pipeline *p, Op &op);
+int op_issue_slots(int opcode);                                   // sm_100a issue slots of one op-IR opcode
 std::vector<std::vector<int>> consumers(const kf_pipeline *p);   // kernel -> consumer kernels
 std::vector<std::vector<int>> producers(const kf_pipeline *p);   // kernel -> producer kernels
 

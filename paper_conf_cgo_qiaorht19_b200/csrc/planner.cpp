@@ -121,7 +121,14 @@ static bool context_legal(const kf_pipeline *p, const std::set<int> &P, const kf
 static double roof_time(const kf_pipeline *p, int ks, int kd, const kf_model_params &m)
 {
     const double ch = p->dtype == KF_U8X4 ? 2.0 : 1.0;
-    auto issue = [&](int k) { const Op &o = p->ops[k]; return (m.c_alu * o.n_alu + m.c_sfu * o.n_sfu) * ch; };
+    auto issue = [&](int k) {
+        const Op &o = p->ops[k];
+        double n = 0.0;
+        for (const Instr &in : o.prog) n += op_issue_slots(in.op);
+        if (o.kind == LOCAL)
+            for (double v : o.mask) n += v != 0.0;
+        return n * ch;
+    };
     std::set<int> ext(p->ops[ks].inputs.begin(), p->ops[ks].inputs.end());
     double slots = issue(ks);
     if (kd >= 0) {
@@ -134,7 +141,8 @@ static double roof_time(const kf_pipeline *p, int ks, int kd, const kf_model_par
         slots = issue(ks) * r + issue(kd);
     }
     const double mem = 4.0 * (double)(ext.size() + 1) / m.bw_bytes_clk;
-    return std::max(mem, slots / m.issue_lanes_clk);
+    const double iss = slots / m.issue_lanes_clk;
+    return std::max(mem, iss) + m.overlap * std::min(mem, iss);
 }
 
 // Benefit of one edge, Eqs. 3-11 plus gamma (Eq. 12 before clamping).

@@ -40,7 +40,7 @@ class ModelParams(C.Structure):
     _fields_ = [("tg", C.c_double), ("ts", C.c_double), ("c_alu", C.c_double), ("c_sfu", C.c_double),
                 ("gamma", C.c_double), ("c_mshared", C.c_double), ("phi_mode", C.c_int32),
                 ("tile_w", C.c_int32), ("tile_h", C.c_int32), ("eq3_mode", C.c_int32),
-                ("bw_bytes_clk", C.c_double), ("issue_lanes_clk", C.c_double)]
+                ("bw_bytes_clk", C.c_double), ("issue_lanes_clk", C.c_double), ("overlap", C.c_double)]
 
 
 class KfError(RuntimeError):

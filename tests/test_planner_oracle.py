@@ -321,18 +321,21 @@ def _chain(prog1, prog2, local2=None, dtype="f32"):
 
 def test_roofline_memory_bound_pair_saves_the_intermediate_image():
     """Two cheap point kernels: each moves 8 B/px unfused, the fused pair 8 B/px,
-    so the benefit is exactly the intermediate's write + read, 2 * 4 B / bw."""
+    so the benefit is exactly the intermediate's write + read, 2 * 4 B / bw
+    (for any overlap: the issue slots of the pair are the sum of its kernels')."""
     m = PL.B200_ROOF_PROFILE
     s = _chain([P.L(0), P.C(1.0), P.ADD], [P.L(0), P.C(2.0), P.MUL])
     info = PL.edge_weights(PL.graph(s), m)
+    # overlap 1: T = M + C, and the pair's issue slots are the sum of its kernels'
     assert info[(0, 1)].w == pytest.approx(8.0 / m.bw_bytes_clk, rel=1e-12)
     assert info[(0, 1)].profitable
 
 
 def test_roofline_issue_bound_pair_gains_nothing():
-    """Two POW-heavy point kernels, each issue-bound alone: fusing saves DRAM time
-    that was hidden anyway, so w = 0 -- unprofitable, an eps edge (Eq. 12, R-3)."""
-    m = PL.B200_ROOF_PROFILE
+    """Two POW-heavy point kernels, each issue-bound alone, under a pure roofline
+    (overlap 0): fusing saves DRAM time that was hidden anyway, so w = 0 --
+    unprofitable, an eps edge (Eq. 12, R-3)."""
+    m = PL.Model(**{**PL.B200_ROOF_PROFILE.__dict__, "overlap": 0.0})
     heavy = [P.L(0), P.C(0.5), P.POW, P.C(0.7), P.POW, P.C(0.9), P.POW]
     s = _chain(heavy, heavy)
     g = PL.graph(s)
@@ -350,15 +353,16 @@ def test_roofline_issue_bound_producer_recompute_costs_its_halo():
     m = PL.B200_ROOF_PROFILE
     heavy = [P.L(0)] + [t for _ in range(15) for t in (P.C(0.99), P.POW)]   # 15 POW: ~600 issue slots / px
     s = _chain(heavy, None, local2=[[1, 1, 1]] * 3)
+    m = PL.Model(**{**m.__dict__, "overlap": 0.0})     # a pure roofline for this limit case
     g = PL.graph(s)
-    n_alu, n_sfu = g.cost[0]
-    i0 = m.c_alu * n_alu + m.c_sfu * n_sfu
+    i0 = 15 * 80.0                                     # 15 POW, 80 issue slots each (kfuse.h)
     fac = (m.tile_w + 2) * (m.tile_h + 2) / (m.tile_w * m.tile_h)
     t0, t1 = PL.roofline_time(g, [0], m), PL.roofline_time(g, [1], m)
     w = PL.edge_weights(g, m)[(0, 1)].w
-    # the consumer alone is memory-bound, the fused pair issue-bound
+    # the consumer alone is memory-bound (9 taps), the fused pair issue-bound
     assert t1 == pytest.approx(8.0 / m.bw_bytes_clk)
-    assert w == pytest.approx(t0 + t1 - (i0 * fac + g.cost[1][0] * m.c_alu) / m.issue_lanes_clk, rel=1e-12)
+    assert t0 == pytest.approx(i0 / m.issue_lanes_clk)
+    assert w == pytest.approx(t0 + t1 - (i0 * fac + 9) / m.issue_lanes_clk, rel=1e-12)
     assert w < 0 and not PL.edge_weights(g, m)[(0, 1)].profitable
 
 
