@@ -214,7 +214,7 @@ def test_full_size_elementwise(cfg):
 
 @pytest.mark.parametrize("wl", ["harris", "deep10", "unsharp"])
 @pytest.mark.parametrize("kind", ["unfused", "paper", "b200"])
-@pytest.mark.parametrize("size", [(300, 200), (64, 1030), (40, 9)])
+@pytest.mark.parametrize("size", [(300, 200), (64, 1030), (40, 9), (130, 1030)])
 def test_run_host_equals_run(wl, kind, size):
     """kf_run_host (row-band pipelined H2D / compute / D2H) == kf_run, bit for bit."""
     spec = P.WORKLOADS[wl](*size)
@@ -361,7 +361,7 @@ def test_c5_full_size_and_bands():
 # ------------------------------------------- halo rows over peer memory (§8(e))
 
 
-def _peer_worker(rank, world, port, wl, graph, q):
+def _peer_worker(rank, world, port, wl, graph, q, width=96):
     import os as _os
     import torch.distributed as dist
     from paper_conf_cgo_qiaorht19_b200 import dist as KD
@@ -369,7 +369,7 @@ def _peer_worker(rank, world, port, wl, graph, q):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         torch.cuda.set_device(0)   # one GPU: the ranks share it, the IPC path is the same as across GPUs
-        spec = P.WORKLOADS[wl](96, 130)
+        spec = P.WORKLOADS[wl](width, 130)
         W, H = spec["width"], spec["height"]
         plan = make_plan(spec, "b200")
         band = KD.partition(H, world, rank, plan.halo_rows)
@@ -436,14 +436,18 @@ def _peer_worker(rank, world, port, wl, graph, q):
     _os2._exit(0)
 
 
-@pytest.mark.parametrize("wl,world,graph", [("harris", 2, False), ("harris", 3, True), ("deep10", 2, True),
-                                             ("two_input", 2, True), ("two_input", 3, False)])
-def test_peer_halo_steps(wl, world, graph):
+@pytest.mark.parametrize("wl,world,graph,width", [("harris", 2, False, 96), ("harris", 3, True, 96),
+                                                   ("deep10", 2, True, 96), ("two_input", 2, True, 96),
+                                                   ("two_input", 3, False, 96), ("harris", 3, True, 130),
+                                                   ("deep10", 2, False, 130)])
+def test_peer_halo_steps(wl, world, graph, width):
     """dist.PeerHalo: halo rows pulled from the neighbours' buffers through CUDA
     IPC mappings, synchronised by device counters (kf_peer_signal / _pull / _wait),
     eager and captured in a CUDA graph, with rotating buffer sets and an
     overwrite guarded by wait_consumed -- bit-identical to the full-image run.
-    The ranks share one GPU here; across GPUs the same mappings are NVLink peers."""
+    Width 130 (not a multiple of 4): unaligned halo rows and band outputs at row
+    offsets.  The ranks share one GPU here; across GPUs the same
+    mappings are NVLink peers."""
     import socket
     import torch.multiprocessing as mp
     sk = socket.socket()
@@ -452,7 +456,7 @@ def test_peer_halo_steps(wl, world, graph):
     sk.close()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_peer_worker, args=(r, world, port, wl, graph, q)) for r in range(world)]
+    procs = [ctx.Process(target=_peer_worker, args=(r, world, port, wl, graph, q, width)) for r in range(world)]
     for p in procs:
         p.start()
     res = {}

@@ -77,6 +77,10 @@ def jobs():
         out.append((P.harris(8, 8, mode), "whole", None, False))
     for wl in ["harris", "deep10", "two_input"]:
         out.append((P.WORKLOADS[wl](96, 130), "b200", None, False))
+        out.append((P.WORKLOADS[wl](130, 130), "b200", None, False))
+    for wl in ["harris", "deep10", "unsharp"]:
+        for kind in ("unfused", "paper", "b200"):
+            out.append((P.WORKLOADS[wl](130, 1030), kind, None, False))
     return out
 
 
