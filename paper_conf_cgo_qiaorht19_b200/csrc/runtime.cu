@@ -18,6 +18,7 @@
 #include <fstream>
 #include <mutex>
 #include <sstream>
+#include <thread>
 
 #include "kf_internal.h"
 #include "device/kf_device.cuh"
@@ -147,7 +148,9 @@ static std::string compile_cubin(const std::string &src, const std::string &name
     nvrtcGetCUBIN(prog, &cubin[0]);
     nvrtcDestroyProgram(&prog);
     mkdir(dir.c_str(), 0775);
-    std::string tmp = path + "." + std::to_string(getpid()) + ".tmp";
+    // per process AND thread: concurrent compiles of the same block write distinct temporaries
+    std::string tmp = path + "." + std::to_string(getpid()) + "." +
+                      std::to_string(std::hash<std::thread::id>()(std::this_thread::get_id())) + ".tmp";
     {
         std::ofstream f(tmp, std::ios::binary);
         if (f) f.write(cubin.data(), (std::streamsize)cubin.size());
