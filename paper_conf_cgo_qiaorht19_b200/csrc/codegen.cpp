@@ -2070,6 +2070,8 @@ const OptDef kOpts[] = {
     {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)
     {"host_taper", 1, 0, 1, false},     // kf_run_host thin first/last bands
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
+    {"st_cs", 0, 0, 1, false},          // streaming (evict-first) 128-bit output stores
+    {"ld_ef", 0, 0, 1, false},          // L2 evict-first hint on the input row copies
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
     {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
     {"persist_waves", 1, 1, 1 << 20, true},
@@ -2288,6 +2290,8 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     o << " } sink " << b.sink << (b.torus ? " (torus)" : "") << "; interior path "
       << (si.ok ? "streaming" : "none") << " (P=" << si.P << " D=" << si.D << " HL=" << si.HL << " L=" << si.L
       << " live~" << si.live_regs << " ops~" << si.iter_ops << (si.rolled ? " rolled" : " unrolled") << ")\n";
+    if (opt(p, "st_cs")) o << "#define KF_ST_CS 1\n";
+    if (opt(p, "ld_ef")) o << "#define KF_LD_EF 1\n";
     o << "#include \"kf_device.cuh\"\n\n";
     for (int k : b.kernels)
         if (!p->ops[k].lut.empty()) {
