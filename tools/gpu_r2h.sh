@@ -9,3 +9,5 @@ $S --config C2 '' 'st_cs=1' 'ld_ef=1' 'st_cs=1 ld_ef=1' >> gpurun_out/sweep_cach
 $S --config C5 --steps 20 '' 'st_cs=1' 'ld_ef=1' 'st_cs=1 ld_ef=1' >> gpurun_out/sweep_cache_r2h.jsonl 2>&1
 $S --config C4 --steps 40 '' 'st_cs=1 ld_ef=1' >> gpurun_out/sweep_cache_r2h.jsonl 2>&1
 cat gpurun_out/sweep_cache_r2h.jsonl
+./tools/ubench/cta_rate > gpurun_out/cta_rate.txt 2>&1 || (cd tools/ubench && nvcc -O3 -gencode arch=compute_100a,code=sm_100a -o cta_rate cta_rate.cu && ./cta_rate > ../../gpurun_out/cta_rate.txt 2>&1)
+cat gpurun_out/cta_rate.txt
