@@ -1745,6 +1745,8 @@ struct StreamGen {
         o << "__device__ __forceinline__ void " << kernel_name(block) << "_fast" << vname(dir, ve, l, r)
           << "(const KfArgs &a, const int chunk, const int strip)\n{\n";
         o << "    const int lane = threadIdx.x & 31;\n";
+        // this warp's private ring (and TMA barriers) in the CTA's shared buffer (option cta_warps)
+        if (si.sring) o << "    const int wslot = (threadIdx.x >> 5) * " << si.warp_smem << ";\n";
         // The image size is fixed per pipeline (one iteration space):
         // baked in, row strides become immediates and unrolled rows use address offsets.
         if (opt(p, "const_w"))
@@ -1812,7 +1814,7 @@ struct StreamGen {
             for (int img : b.ext) {
                 int s = slot.at(img);
                 o << "    " << (f32 ? "float4" : "uint4") << " *sr" << s << " = (" << (f32 ? "float4" : "uint4")
-                  << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 * NQ << ") + lane * " << NQ << ";\n";
+                  << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 * NQ << " + wslot) + lane * " << NQ << ";\n";
             }
             if (tma) {
                 // one mbarrier per (image, ring slot) after the rings.  The warp's
@@ -1821,7 +1823,7 @@ struct StreamGen {
                 // pointer already starts at the clipped column max(x0w, 0), which
                 // lands at byte toff of the slot.  Lanes wholly outside the image
                 // keep stale ring data: they are halo lanes no stored pixel reads.
-                o << "    unsigned long long *mb = (unsigned long long *)(" << kernel_name(block) << "_smem + "
+                o << "    unsigned long long *mb = (unsigned long long *)(" << kernel_name(block) << "_smem + wslot + "
                   << si.ring_bytes << ");\n";
                 o << "    const int x0w = a.fx0 + (chunk * " << 32 - 2 * HL << " - " << HL << ") * " << V << ";\n";
                 o << "    const unsigned toff = (unsigned)(max(x0w, 0) - x0w) * 4u;\n";
@@ -2070,8 +2072,7 @@ const OptDef kOpts[] = {
     {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)
     {"host_taper", 1, 0, 1, false},     // kf_run_host thin first/last bands
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
-    {"st_cs", 0, 0, 1, false},          // streaming (evict-first) 128-bit output stores
-    {"ld_ef", 0, 0, 1, false},          // L2 evict-first hint on the input row copies
+    {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
     {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
     {"persist_waves", 1, 1, 1 << 20, true},
@@ -2276,6 +2277,9 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     si.edge_l = !rep && hfit && p->W >= 4 * kV_;
     si.edge_r = si.edge_l && si.vec;
     si.ok = b.Rx <= 2 * kV_ * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
+    si.warp_smem = (si.ring_bytes + (si.tma ? 8 * (int)b.ext.size() * si.DS : 0) + 15) / 16 * 16;
+    // warps per CTA, capped so the CTA's static shared buffer stays within 48 KB
+    si.nw = std::max(1, std::min((int)opt(p, "cta_warps"), 49152 / std::max(si.warp_smem, 1)));
     if (opt(p, "naive_border")) si.ok = false;   // negative control: everything through the (naive) frame
     return si;
 }
@@ -2290,8 +2294,6 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     o << " } sink " << b.sink << (b.torus ? " (torus)" : "") << "; interior path "
       << (si.ok ? "streaming" : "none") << " (P=" << si.P << " D=" << si.D << " HL=" << si.HL << " L=" << si.L
       << " live~" << si.live_regs << " ops~" << si.iter_ops << (si.rolled ? " rolled" : " unrolled") << ")\n";
-    if (opt(p, "st_cs")) o << "#define KF_ST_CS 1\n";
-    if (opt(p, "ld_ef")) o << "#define KF_LD_EF 1\n";
     o << "#include \"kf_device.cuh\"\n\n";
     for (int k : b.kernels)
         if (!p->ops[k].lut.empty()) {
@@ -2308,8 +2310,8 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
             n = std::max(n, (kFrameTiles[s][0] + 2 * b.hx.at(k)) * (kFrameTiles[s][1] + 2 * b.hy.at(k)));
         frame_bytes += n * 4;
     }
-    const int ring_total = si.ring_bytes + (si.tma ? 8 * (int)b.ext.size() * si.DS : 0);   // + TMA mbarriers
-    const int smem_bytes = std::max(16, std::max(frame_bytes, si.ok && si.sring ? ring_total : 0));
+    const int NW = si.nw;   // interior warps per CTA (option cta_warps): one ring each
+    const int smem_bytes = std::max(16, std::max(frame_bytes, si.ok && si.sring ? NW * si.warp_smem : 0));
     o << "__shared__ __align__(16) unsigned char " << kernel_name(block) << "_smem[" << smem_bytes << "];\n\n";
     FrameGen fg(p, b, block, o);
     fg.run();
@@ -2317,7 +2319,8 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
         StreamGen sg(p, b, si, block, o);
         sg.run();
     }
-    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads << ", " << opt(p, "minctas") << ") " << kernel_name(b, block)
+    o << "extern \"C\" __global__ void __launch_bounds__(" << kThreads * NW << ", "
+      << std::max(1, (int)opt(p, "minctas") / NW) << ") " << kernel_name(b, block)
       << "(const __grid_constant__ KfArgs a)\n{\n";
     // Persistent CTAs: the grid is at most one wave of resident CTAs, and each
     // loops over work items (frame tiles first, then interior items) with a
@@ -2325,11 +2328,22 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     // and the trip count are CTA-uniform, so the warp shuffles of the interior
     // path need no convergence barriers.  No cp.async copy is in flight between
     // items (every issued row was waited for), so the shared ring is reused.
-    o << "    const int total = a.frame_ctas + a.n_items;\n";
+    // With NW > 1 warps per CTA a frame unit uses all of them (its loops stride
+    // by blockDim), an interior unit gives each warp its own item and ring.
+    o << "    const int total = a.frame_ctas + (a.n_items + " << NW - 1 << ") / " << NW << ";\n";
     o << "    for (int cta = blockIdx.x; cta < total; cta += gridDim.x) {\n";
     o << "        if (cta < a.frame_ctas) " << kernel_name(block) << "_frame(a, cta);\n";
-    if (si.ok) o << "        else " << kernel_name(block) << "_fast(a, cta - a.frame_ctas);\n";
-    o << "        __syncwarp();\n";
+    if (si.ok) {
+        if (NW == 1) {
+            o << "        else " << kernel_name(block) << "_fast(a, cta - a.frame_ctas);\n";
+        } else {
+            o << "        else {\n";
+            o << "            const int item = (cta - a.frame_ctas) * " << NW << " + (int)(threadIdx.x >> 5);\n";
+            o << "            if (item < a.n_items) " << kernel_name(block) << "_fast(a, item);\n";
+            o << "        }\n";
+        }
+    }
+    o << (NW == 1 ? "        __syncwarp();\n" : "        __syncthreads();\n");
     o << "    }\n";
     o << "}\n";
     return o.str();

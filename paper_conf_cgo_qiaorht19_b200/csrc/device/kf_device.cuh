@@ -189,30 +189,13 @@ __device__ __forceinline__ void kf_sti(void *p, int base, int W, int y, int x, I
 // 128-bit accesses of the streaming path (4 pixels per lane)
 __device__ __forceinline__ float4 kf_ld4f(const float *p) { return __ldg((const float4 *)p); }
 __device__ __forceinline__ uint4 kf_ld4u(const unsigned *p) { return __ldg((const uint4 *)p); }
-// Cache policy of the streaming path (schedule options st_cs / ld_ef, set by
-// the generated kernel before this header): streaming stores (st.global.cs,
-// evict first) and an L2 evict-first hint on the input row copies.
-#ifndef KF_ST_CS
-#define KF_ST_CS 0
-#endif
-#ifndef KF_LD_EF
-#define KF_LD_EF 0
-#endif
 __device__ __forceinline__ void kf_st4f(float *p, float a, float b, float c, float d)
 {
-#if KF_ST_CS
-    __stcs((float4 *)p, make_float4(a, b, c, d));
-#else
     *(float4 *)p = make_float4(a, b, c, d);
-#endif
 }
 __device__ __forceinline__ void kf_st4u(unsigned *p, unsigned a, unsigned b, unsigned c, unsigned d)
 {
-#if KF_ST_CS
-    __stcs((uint4 *)p, make_uint4(a, b, c, d));
-#else
     *(uint4 *)p = make_uint4(a, b, c, d);
-#endif
 }
 #define KF_FULL 0xffffffffu
 __device__ __forceinline__ float kf_shup(float v, int d) { return __shfl_up_sync(KF_FULL, v, d); }
@@ -289,14 +272,7 @@ __device__ __forceinline__ F2 kf2_sel_gt(F2 a, F2 b, F2 c, F2 d)
 __device__ __forceinline__ void kf_cp16(void *smem, const void *gmem)
 {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-#if KF_LD_EF
-    unsigned long long pol;
-    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(pol));
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "l"(pol)
-                 : "memory");
-#else
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
-#endif
 }
 __device__ __forceinline__ void kf_cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N> __device__ __forceinline__ void kf_cp_wait()

@@ -148,6 +148,8 @@ struct StreamInfo {
     int live_regs = 0;            // estimate of ring registers
     bool rolled = false;          // one loop-body copy + ring shifts (big blocks)
     int T = 1;                    // rows per rolled trip (body copies per rolled loop trip)
+    int nw = 1;                   // interior warps per CTA (option cta_warps)
+    int warp_smem = 0;            // shared-memory bytes of one warp's ring (+ TMA barriers)
     bool sring = false;           // external rows fed by a cp.async shared-memory ring
     int DS = 0;                   // rows in that ring (multiple of P)
     bool lpf = false;             // ring rows read one iteration ahead (LDS latency off the critical path)

@@ -224,7 +224,8 @@ void prepare(kf_pipeline *p, kf_plan *plan)
             cu_check(d.moduleGetFunction(&cb->fn, cb->mod, kernel_name(plan->info[i], (int)i).c_str()), "cuModuleGetFunction");
             cb->source = src;
             cb->si = stream_info(p, plan->info[i]);
-            cu_check(d.occupancy(&cb->ctas_per_sm, cb->fn, kThreads, 0), "cuOccupancyMaxActiveBlocksPerMultiprocessor");
+            cu_check(d.occupancy(&cb->ctas_per_sm, cb->fn, kThreads * cb->si.nw, 0),
+                     "cuOccupancyMaxActiveBlocksPerMultiprocessor");
             cb->ctas_per_sm = std::max(1, cb->ctas_per_sm);
             KF_CUDA(cudaDeviceGetAttribute(&cb->num_sms, cudaDevAttrMultiProcessorCount, dev));
             it = p->rt->modules.emplace(h, cb).first;
@@ -301,7 +302,7 @@ static unsigned launch_geometry(const kf_pipeline *p, KfArgs &a, const BlockInfo
     const int chunk_w = (32 - 2 * si.HL) * V;
     a.n_chunks = (fx1 - fx0 + chunk_w - 1) / chunk_w;
     const int Hf = fy1 - fy0;
-    const long long slots = (long long)cb.num_sms * cb.ctas_per_sm;   // resident single-warp CTAs per wave
+    const long long slots = (long long)cb.num_sms * cb.ctas_per_sm * si.nw;   // resident interior warps per wave
     // ns balanced strips of floor/ceil(Hf/ns) rows.  Edge strips must be at
     // least L rows so that no interior strip reads beyond the image; a top and
     // a bottom edge need two strips.  Cost (fitted to B200 sweeps, DESIGN.md
@@ -336,7 +337,7 @@ static unsigned launch_geometry(const kf_pipeline *p, KfArgs &a, const BlockInfo
         if (n > 0 && Hf / (best_ns + n) >= smin) a.n_long = n;
     }
     a.n_items = a.n_chunks * a.n_strips;
-    return (unsigned)(cta + a.n_items);
+    return (unsigned)(cta + (a.n_items + si.nw - 1) / si.nw);   // si.nw interior items per CTA
 }
 
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
@@ -427,7 +428,7 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         }
         if (grid == 0) continue;
         void *params[] = {&a};
-        cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
+        cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads * cb.si.nw, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
     }
     for (auto &c : band_copies) {
         const char *src = (const char *)plan->workspace[c.first] + (size_t)row0 * p->W * 4;

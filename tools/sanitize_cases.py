@@ -54,6 +54,10 @@ def main():
             run(P.deep10(45, 37, mode), "b200")
             n += 2
         run(P.harris(256, 256), "b200", {"tma": 1})
+        run(P.harris(256, 256), "b200", {"cta_warps": 4})
+        run(P.deep10(67, 41), "b200", {"cta_warps": 4})
+        run(P.harris(45, 37, "constant"), "b200", {"cta_warps": 4})
+        n += 3
         run(P.unsharp(512, 96), "b200", {"tma": 1})
         n += 2
         plan, ins, outs = run(P.harris(300, 200), "b200")
