@@ -1746,7 +1746,12 @@ struct StreamGen {
           << "(const KfArgs &a, const int chunk, const int strip)\n{\n";
         o << "    const int lane = threadIdx.x & 31;\n";
         // this warp's private ring (and TMA barriers) in the CTA's shared buffer (option cta_warps)
-        if (si.sring) o << "    const int wslot = (threadIdx.x >> 5) * " << si.warp_smem << ";\n";
+        if (si.sring) {
+            if (si.nw > 1)
+                o << "    const int wslot = (threadIdx.x >> 5) * " << si.warp_smem << ";\n";
+            else
+                o << "    constexpr int wslot = 0;\n";
+        }
         // The image size is fixed per pipeline (one iteration space):
         // baked in, row strides become immediates and unrolled rows use address offsets.
         if (opt(p, "const_w"))
