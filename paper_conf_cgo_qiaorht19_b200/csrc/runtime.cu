@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nvrtc.h>
+#include <nvtx3/nvToolsExt.h>
 #include <sys/stat.h>
 #include <utime.h>
 #include <unistd.h>
@@ -24,6 +25,13 @@
 #include "device/kf_device.cuh"
 
 namespace kf {
+
+// NVTX ranges around the host-side steps (prepare, run, run_host and its
+// bands): visible in Nsight Systems / ncu range filters, free without a tool.
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 static const char *kDeviceHeader =
 #include "kf_device_cuh.inc"
@@ -206,6 +214,7 @@ std::string compile_block_cubin(const kf_pipeline *p, const kf_plan *plan, int i
 void prepare(kf_pipeline *p, kf_plan *plan)
 {
     if (plan->prepared) return;
+    NvtxRange nvtx("kf_prepare");
     Driver &d = driver();
     if (!p->rt) p->rt = new Runtime();
     int dev = 0;
@@ -361,6 +370,7 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
     prepare(p, plan);
     Driver &d = driver();
     const bool band = !(row0 == 0 && row1 == p->H && in_row0 == 0);
+    NvtxRange nvtx(band ? "kf_run_band" : "kf_run");
     const int nimg = p->n_images();
     // rows each image must be available over
     std::vector<int> lo(nimg, INT32_MAX), hi(nimg, INT32_MIN);
@@ -450,6 +460,7 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
 {
     if (n_in != p->n_inputs || n_out != (int)p->outputs.size()) fail(KF_ERR_ARG, "wrong number of buffers");
     prepare(p, plan);
+    NvtxRange nvtx("kf_run_host");
     Runtime &rt = *p->rt;
     const size_t row_bytes = (size_t)p->W * 4, bytes = row_bytes * p->H;
     if (rt.stage_bytes != bytes || rt.stage_in.size() != (size_t)n_in || rt.stage_out.size() != (size_t)n_out) {
