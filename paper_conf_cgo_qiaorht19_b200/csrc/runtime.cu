@@ -180,7 +180,7 @@ struct CompiledBlock {
     }
 };
 
-constexpr int kHostBands = 8;   // kf_run_host pipeline depth (row bands; 16 measured slower)
+constexpr int kHostBands = 32;  // kf_run_host: most row bands (option host_bands, default 8)
 
 struct Runtime {
     std::map<uint64_t, std::shared_ptr<CompiledBlock>> modules;   // by source hash
@@ -488,7 +488,8 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     bool repeat = false;
     for (const auto &op : p->ops) repeat |= op.kind == LOCAL && op.mode == KF_REPEAT;
     const int R = plan->halo_rows;
-    int nb = repeat ? 1 : std::max(1, std::min(kHostBands, p->H / std::max(64, 4 * R)));
+    const int want = std::min(kHostBands, (int)opt(p, "host_bands"));
+    int nb = repeat ? 1 : std::max(1, std::min(want, p->H / std::max(64, 4 * R)));
     std::vector<const void *> din(rt.stage_in.begin(), rt.stage_in.end());
     // the copy streams start after everything already queued on the caller's stream
     KF_CUDA(cudaEventRecord(rt.ev_start, s));
@@ -498,11 +499,16 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     // Band boundaries.  Only the first band's upload and the last band's
     // download are exposed (everything else overlaps), so with 8 bands the
     // ends are thin: row shares 1,3,6,6,6,6,3,1 / 32 (uniform when fewer bands).
-    static const int kShare8[9] = {0, 1, 4, 10, 16, 22, 28, 31, 32};
+    // Tapered shares (option host_taper, nb >= 5): 1, 3, 6, ..., 6, 3, 1 units
+    // (nb = 8: 1,3,6,6,6,6,3,1 / 32), else uniform.
+    const bool taper = nb >= 5 && opt(p, "host_taper");
+    auto units = [&](int k) { return !taper ? 1 : (k == 0 || k == nb - 1) ? 1 : (k == 1 || k == nb - 2) ? 3 : 6; };
+    long long tot_units = 0;
+    for (int k = 0; k < nb; k++) tot_units += units(k);
     auto cut = [&](int k) {
-        if (nb == kHostBands && kHostBands == 8 && opt(p, "host_taper"))
-            return (int)((long long)p->H * kShare8[k] / 32);
-        return (int)((long long)p->H * k / nb);
+        long long u = 0;
+        for (int i = 0; i < k; i++) u += units(i);
+        return (int)((long long)p->H * u / tot_units);
     };
     for (int k = 0; k < nb; k++) {
         const int r0 = cut(k), r1 = cut(k + 1);
