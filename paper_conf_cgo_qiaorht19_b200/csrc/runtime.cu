@@ -461,6 +461,33 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     if (n_in != p->n_inputs || n_out != (int)p->outputs.size()) fail(KF_ERR_ARG, "wrong number of buffers");
     prepare(p, plan);
     NvtxRange nvtx("kf_run_host");
+    if (opt(p, "host_direct")) {
+        // Zero-copy (option host_direct): when every host buffer is pinned and
+        // mapped (UVA: cudaHostAlloc / torch pin_memory), the kernels read the
+        // inputs and write the outputs over the host link directly -- no staging
+        // copies, no band pipeline.  Otherwise the staged path below runs.
+        std::vector<const void *> di(n_in);
+        std::vector<void *> dq(n_out);
+        bool ok = true;
+        auto mapped = [&](const void *h, void **d) {
+            cudaPointerAttributes at;
+            if (cudaPointerGetAttributes(&at, h) != cudaSuccess) { cudaGetLastError(); return false; }
+            if (at.type != cudaMemoryTypeHost || !at.devicePointer) return false;
+            *d = at.devicePointer;
+            return true;
+        };
+        for (int i = 0; i < n_in && ok; i++) {
+            void *d = nullptr;
+            ok = mapped(hin[i], &d);
+            di[i] = d;
+        }
+        for (int j = 0; j < n_out && ok; j++) ok = mapped(hout[j], &dq[j]);
+        if (ok) {
+            run(p, plan, di.data(), n_in, dq.data(), n_out, stream, 0, p->H, 0, p->H);
+            KF_CUDA(cudaStreamSynchronize((cudaStream_t)stream));
+            return;
+        }
+    }
     Runtime &rt = *p->rt;
     const size_t row_bytes = (size_t)p->W * 4, bytes = row_bytes * p->H;
     if (rt.stage_bytes != bytes || rt.stage_in.size() != (size_t)n_in || rt.stage_out.size() != (size_t)n_out) {

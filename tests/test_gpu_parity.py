@@ -226,6 +226,23 @@ def test_run_host_equals_run(wl, kind, size):
     np.testing.assert_array_equal(out, dev)
 
 
+@pytest.mark.parametrize("opts", [{"host_bands": 1}, {"host_bands": 3}, {"host_bands": 16}, {"host_bands": 32},
+                                  {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}])
+def test_run_host_pipeline_depth_bit_identical(opts):
+    """Any kf_run_host band count / taper (options host_bands, host_taper) gives
+    kf_run's bits (each band is a kf_run_band with global border handling)."""
+    spec = P.harris(130, 1030)
+    ins = _inputs(spec, 14)
+    dev = run_gpu(spec, make_plan(spec, "b200"), ins)[0]
+    out = np.empty_like(dev)
+    make_plan(spec, "b200", opts).run_host([np.ascontiguousarray(ins[0])], [out])   # pageable: staged path
+    np.testing.assert_array_equal(out, dev)
+    hin = torch.from_numpy(np.ascontiguousarray(ins[0])).pin_memory()               # pinned: direct if asked
+    hout = torch.zeros(dev.shape, dtype=torch.float32).pin_memory()
+    make_plan(spec, "b200", opts).run_host([hin], [hout])
+    np.testing.assert_array_equal(hout.numpy(), dev)
+
+
 def test_run_host_repeat_and_pinned():
     """REPEAT plans (one band) and pinned host buffers on a non-default stream."""
     spec = P.harris(256, 300, "repeat")
