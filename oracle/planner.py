@@ -19,10 +19,15 @@ Contents, each in the paper's notation:
                   comparison column of Table I,
                   reading R-18
 
-Parity unpinned (R-4, R-7): the local-to-local locality gain of Eq. 3
-(garbled, read as IS*tg/ts) and the B200 profile's STAGED recompute factor have
-no numeric example in the paper; only the point-based / point-to-local weights
-(328/256/eps) and the Eq. 9 sizes are pinned.
+What pins what (R-4, R-7, R-20): the point-based / point-to-local
+weights (328/256/eps) and the Eq. 9 sizes are the paper's
+numbers; the B200 profile's STAGED recompute factor (R-4) is pinned by its two
+reductions (a 1x1 tile gives Eq. 7 and the paper's 328/256; an unbounded tile
+gives no recompute); the ROOFLINE weights (R-20) by their limit cases.  Parity
+unpinned: the VALUE of the local-to-local locality gain of Eq. 3 (garbled, read
+as IS*tg/ts, R-7) -- the paper gives no number for it, only the sign in the
+Night filter (an unprofitable local-to-local pair), which
+is pinned.
 
 Weights are lexicographic pairs (real, eps-count) with the real part in fixed
 point q = floor(w * 2^20 + 0.5) (reading O1-i): sums are exact, so ties

@@ -285,3 +285,15 @@ def test_library_reads_no_environment():
     assert not [t for t in strings if t.startswith("KFUSE_") and t != "KFUSE_CACHE_DIR"], \
         [t for t in strings if t.startswith("KFUSE_")]
     assert "getenv" in syms
+
+
+def test_staged_profile_reductions_through_the_abi():
+    """The product planner's STAGED factor (R-4) reduces to the paper's Eq. 7 at a
+    1x1 tile (Harris 328 / 256) and to no recompute at an
+    unbounded tile (400 - 8 = 392)."""
+    spec = P.harris(64, 64)
+    ix = {o["name"]: k for k, o in enumerate(spec["ops"])}
+    one = K.Pipeline.from_spec(spec).plan_fusion(K.model_params("b200", tile_w=1, tile_h=1))
+    assert one.edge(ix["sx"], ix["gx"])["w"] == 328.0 and one.edge(ix["sxy"], ix["gxy"])["w"] == 256.0
+    big = K.Pipeline.from_spec(spec).plan_fusion(K.model_params("b200", tile_w=1 << 20, tile_h=1 << 20))
+    assert abs(big.edge(ix["sx"], ix["gx"])["w"] - 392.0) < 1e-3

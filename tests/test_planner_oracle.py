@@ -378,3 +378,29 @@ def test_roofline_plan_bounded_by_bruteforce(seed):
     for b in pl.blocks:
         assert PL.is_legal(g, set(b), m, pl.info)
     assert pl.beta <= PL.brute_force(s, m)[0]
+
+
+# --------------------------------- STAGED recompute factor (R-4) reductions
+
+def _staged(tile):
+    return PL.Model(c_mshared=5.0, phi_mode=1, tile_w=tile, tile_h=tile)
+
+
+def test_staged_factor_one_pixel_tile_is_the_papers_per_tap_recompute(harris):
+    """R-4 reduces to the paper: with a 1x1 staged tile every consumer pixel
+    recomputes its producer on the whole mask footprint, (1+2rx)(1+2ry) = sz(kd),
+    i.e. Eq. 7 -- so the point-to-local Harris weights become the worked
+    example's 328 / 256."""
+    pl = PL.get_legal_partitions(harris, _staged(1))
+    w = {tuple(names(harris, k)): e.w for k, e in pl.info.items()}
+    assert w[("sx", "gx")] == 328.0 and w[("sy", "gy")] == 328.0 and w[("sxy", "gxy")] == 256.0
+
+
+def test_staged_factor_infinite_tile_recomputes_nothing(harris):
+    """The other end of R-4: as the staged tile grows, the halo share vanishes and
+    the producer is computed once per pixel, phi -> costop * IS_ks:
+    w(sx, gx) -> tg - cALU*nALU*1 = 400 - 8 = 392, w(sxy, gxy) -> 400 - 16 = 384."""
+    pl = PL.get_legal_partitions(harris, _staged(1 << 20))
+    w = {tuple(names(harris, k)): e.w for k, e in pl.info.items()}
+    assert w[("sx", "gx")] == pytest.approx(392.0, abs=1e-3)
+    assert w[("sxy", "gxy")] == pytest.approx(384.0, abs=1e-3)
