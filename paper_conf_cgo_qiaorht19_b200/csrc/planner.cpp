@@ -135,8 +135,8 @@ static double roof_time(const kf_pipeline *p, int ks, int kd, const kf_model_par
         const Op &d = p->ops[kd];
         for (int i : d.inputs)
             if (i != p->n_inputs + ks) ext.insert(i);
-        const double r = d.kind == LOCAL ? (double)((m.tile_w + 2 * d.rx()) * (m.tile_h + 2 * d.ry())) /
-                                                   (double)(m.tile_w * m.tile_h)
+        const double r = d.kind == LOCAL ? ((double)(m.tile_w + 2 * d.rx()) * (double)(m.tile_h + 2 * d.ry())) /
+                                                   ((double)m.tile_w * (double)m.tile_h)
                                          : 1.0;
         slots = issue(ks) * r + issue(kd);
     }
@@ -167,7 +167,8 @@ static EdgeInfo benefit(const kf_pipeline *p, int ks, int kd, const kf_model_par
     }
     double fac;
     if (m.phi_mode == 1)                                      // STAGED (R-4)
-        fac = (double)((m.tile_w + 2 * d.rx()) * (m.tile_h + 2 * d.ry())) / (double)(m.tile_w * m.tile_h);
+        fac = ((double)(m.tile_w + 2 * d.rx()) * (double)(m.tile_h + 2 * d.ry())) /
+              ((double)m.tile_w * (double)m.tile_h);   // in double: large tiles must not overflow int
     else if (s.kind == POINT)
         fac = (double)((2 * d.rx() + 1) * (2 * d.ry() + 1)); // sz(kd), Eq. 7
     else
