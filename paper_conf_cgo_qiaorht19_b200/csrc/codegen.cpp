@@ -1865,7 +1865,11 @@ struct StreamGen {
         // peeled iterations: the 2L warm-up iterations (only the kernels whose rows
         // are needed run) and, at an image edge, those in which some tap row lies
         // beyond the edge (remapped statically)
-        int need = si.rolled ? 0 : 2 * L;
+        // option peel_warmup = 0: an unrolled body runs its 2L warm-up iterations
+        // through the loop itself (every kernel computed, stores masked) instead
+        // of a peeled prologue that computes only the kernels already needed --
+        // more arithmetic, less straight-line code (edge strips still peel)
+        int need = si.rolled || !opt(p, "peel_warmup") ? 0 : 2 * L;
         vedge = ve;
         if (ve)
             for (int k : b.kernels)
@@ -2070,6 +2074,7 @@ const OptDef kOpts[] = {
     {"qptr", 1, 0, 1, false},           // per-trip ring slot base pointers
     {"heavy_first", 1, 0, 1, false},    // edge items first
     {"code_budget", 12000, 0, 1 << 30, false},   // unrolled vs rolled body
+    {"peel_warmup", 1, 0, 1, false},    // unrolled bodies peel the 2L warm-up iterations
     {"rtrip", 1, 1, 2, false},          // rows per trip of a rolled body (2: half the ring moves, but
                                         // twice the loop code: measured slower, instruction fetch stalls)
     {"rolled_edge_v", 1, 0, 1, false},  // rolled bodies keep the edge strips

@@ -54,7 +54,8 @@ def jobs():
             {"sring": 0}, {"minctas": 8}, {"code_budget": 1000}, {"swring": 0}, {"tma": 1},
             {"tma": 1, "lds_pf": 0}, {"tma": 1, "code_budget": 1000}, {"tma": 1, "smem_rows": 6}, {"rtrip": 2},
             {"rtrip": 2, "code_budget": 1000}, {"code_budget": 1000, "lds_pf": 0}, {"cta_warps": 2},
-            {"cta_warps": 4}, {"cta_warps": 8}, {"cta_warps": 4, "tma": 1}, {"cta_warps": 4, "code_budget": 1000}]
+            {"cta_warps": 4}, {"cta_warps": 8}, {"cta_warps": 4, "tma": 1}, {"cta_warps": 4, "code_budget": 1000},
+            {"peel_warmup": 0}, {"peel_warmup": 0, "lds_pf": 0}]
     exp = [{"v8": 1}, {"persist": 1}, {"nlong": 3}]
     for wl in ["harris", "unsharp", "shitomasi"]:
         for o in ({"pairs": 0}, {"defer": 0}):
@@ -64,7 +65,7 @@ def jobs():
         out.append((spec, "b200", {"tma": 1}, False))
     out.append((P.copy(4096, 4096), "b200", {"tma": 1}, False))
     out.append((P.copy(4096, 4096), "b200", None, False))
-    for o in ({"cta_warps": 2}, {"cta_warps": 4}, {"cta_warps": 8}):
+    for o in ({"peel_warmup": 0},):
         for cfg in ("C2", "C3", "C3s", "C4", "C5"):
             out.append((P.config(cfg)[0], "b200", o, False))
         out.append((P.copy(4096, 4096), "b200", o, False))
