@@ -1,4 +1,5 @@
-"""Small launches of every kernel family for compute-sanitizer (tools/sanitize.sh):
+"""TEST INFRASTRUCTURE (not collected by pytest): small launches of every kernel
+family for compute-sanitizer (tools/sanitize.sh):
 C1 Harris 256^2 under every plan, deep10 67x41, all five border modes fused
 (Harris and deep10), 10 random DAGs (3 plans each), the TMA row feed, kf_run_host
 and a row band.  Each result is also checked against the oracle, so a run under
@@ -7,7 +8,7 @@ import os
 import random
 import sys
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))   # tests/ -> repo root
 sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402

@@ -9,4 +9,4 @@ for cfg in C4 C3; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:kf_b -s 2 -c 1 -f -o gpurun_out/r02_${cfg}_b200_full \
      python tools/prof_run.py --config $cfg --plan b200 > gpurun_out/ncu_${cfg}.log 2>&1; echo "ncu $cfg rc=$?"
 done
-timeout 600 /usr/local/cuda/bin/compute-sanitizer --tool memcheck --error-exitcode 9 python tools/sanitize_cases.py peer > gpurun_out/sanitize_peer1.log 2>&1; echo "sanitize peer rc=$?"; tail -2 gpurun_out/sanitize_peer1.log
+timeout 600 /usr/local/cuda/bin/compute-sanitizer --tool memcheck --error-exitcode 9 python tests/sanitize_cases.py peer > gpurun_out/sanitize_peer1.log 2>&1; echo "sanitize peer rc=$?"; tail -2 gpurun_out/sanitize_peer1.log
