@@ -22,6 +22,23 @@ PW_TOL = 1e-3   # pointwise relative error on pixels with |oracle| >= PW_FLOOR *
 PW_FLOOR = 1e-3  # DESIGN R-17: f32 rounding of the largest term, ~4 ulp * max|term|, is <= 2.4e-4 there)
 
 
+@pytest.fixture(scope="module", autouse=True)
+def _precompile_kernels():
+    """Compiles every kernel this module launches up front, in parallel threads
+    (NVRTC releases the GIL): instant when the in-tree cubin cache is warm (build()
+    warms it), a few minutes instead of a serial compile per test when it is not."""
+    import importlib.util
+    import os
+    from concurrent.futures import ThreadPoolExecutor
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    spec = importlib.util.spec_from_file_location("warm_test_cache", os.path.join(root, "tools", "warm_test_cache.py"))
+    w = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(w)
+    with ThreadPoolExecutor(max(1, min(32, os.cpu_count() or 1))) as ex:
+        list(ex.map(w.compile_job, w.jobs()))
+    yield
+
+
 def _inputs(spec, seed):
     return [gen.image(spec["dtype"], seed + 101 * j, spec["width"], spec["height"]) for j in range(spec["n_inputs"])]
 
