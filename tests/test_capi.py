@@ -214,6 +214,15 @@ def test_exact_planner_equals_bruteforce_on_random_dags(seed):
     _check_exact(spec, rng.choice(["paper", "b200"]))
 
 
+@pytest.mark.parametrize("seed", range(20))
+def test_exact_planner_equals_bruteforce_roofline(seed):
+    """kf_plan_exact under the ROOFLINE weights (R-20) = the brute-force optimum of
+    the independent Python planner, and Alg. 1 never beats it."""
+    rng = random.Random(9700 + seed)
+    spec = P.random_pipeline(rng, 16, 16, rng.choice(["f32", "u8x4"]), rng.randint(1, 7))
+    _check_exact(spec, "b200roof")
+
+
 def test_exact_planner_beats_min_cut_counterexample():
     """Alg. 1 reaches 350 on the 5-local chain, the optimum is 550."""
     p = P.Pipeline("chain", 32, 32, "f32")

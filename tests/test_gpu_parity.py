@@ -322,6 +322,33 @@ def test_overlapped_step_equals_full_run(wl, rank, world, monkeypatch):
     np.testing.assert_array_equal(out.cpu().numpy(), full[band.row0:band.row1])
 
 
+@pytest.mark.parametrize("wl", ["harris", "deep10"])
+def test_run_is_graph_capturable(wl):
+    """kf_run on a side stream captured into a CUDA graph (as bench.py times it):
+    replays reproduce the eager result, on rotating buffers."""
+    spec = P.WORKLOADS[wl](300, 200)
+    ins = [_inputs(spec, 30 + k) for k in range(2)]
+    plan = make_plan(spec, "b200")
+    ref = [run_gpu(spec, plan, i)[0] for i in ins]
+    d_in = [[torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in i] for i in ins]
+    outs = [_alloc(spec) for _ in ins]
+    s = torch.cuda.Stream()
+    plan.run(d_in[0], outs[0], s)      # prepare + warm up outside the capture
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for k in (0, 1):
+            plan.run(d_in[k], outs[k], s)
+    for o in outs:
+        o[0].zero_()
+    with torch.cuda.stream(s):
+        g.replay()
+        g.replay()
+    torch.cuda.synchronize()
+    for k in (0, 1):
+        np.testing.assert_array_equal(outs[k][0].cpu().numpy(), ref[k])
+
+
 def test_launch_count_matches_blocks():
     spec = P.harris(512, 512)
     for kind, n in (("unfused", 9), ("paper", 6), ("b200", 1)):
