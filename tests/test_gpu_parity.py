@@ -672,3 +672,14 @@ def test_negative_control_pad_once_fails_parity(wl, mode):
     if wl == "fig4" and mode == "clamp":
         assert naive[0, 0] == 684 and good[0, 0] == 763
     _log_parity(test="negative_control", workload=wl, mode=mode, pixels=int(bad.size), failing=int(bad.sum()))
+
+
+def test_c_abi_run_from_plain_c(tmp_path):
+    """examples/harris_c.c runs the fused plan through kf_run_host from plain C."""
+    import subprocess
+    import sys
+    sys.path.insert(0, __import__("os").path.dirname(__file__))
+    from test_capi import _build_c_example
+    r = subprocess.run([_build_c_example(tmp_path), "run"], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
+    assert "ran the fused plan on 512x384" in r.stdout
