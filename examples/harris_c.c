@@ -77,6 +77,7 @@ int main(int argc, char **argv)
            (int)kf_plan_num_launches(pb), (int)kf_plan_halo_rows(pb));
 
     int rc = 0;
+    if (argc > 1 && !strcmp(argv[1], "compile")) CHECK(kf_compile_plan(p, pb));   /* NVRTC only, no GPU */
     if (argc > 1 && !strcmp(argv[1], "run")) {
         float *h_in = (float *)malloc(sizeof(float) * W * H), *h_out = (float *)malloc(sizeof(float) * W * H);
         for (int i = 0; i < W * H; i++) h_in[i] = (float)((i * 2654435761u) >> 8 & 0xffff) / 65536.0f;
