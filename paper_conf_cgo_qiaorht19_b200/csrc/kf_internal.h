@@ -5,6 +5,7 @@
 #include <map>
 #include <memory>
 #include <set>
+#include <tuple>
 #include <string>
 #include <vector>
 
@@ -87,6 +88,13 @@ struct BlockInfo {
 };
 
 struct CompiledBlock;             // runtime.cu
+// Memoised launch geometry of one block launch (runtime.cu): the geometry tail
+// of the kernel arguments (frame rectangles onward) and the grid size.
+struct Geom {
+    std::vector<unsigned char> tail;
+    unsigned grid = 0;
+};
+using GeomKey = std::tuple<int, int, int, long long, long long>;   // block, rows [r0, r1), nstrips, nlong
 
 }  // namespace kf
 
@@ -101,6 +109,7 @@ struct kf_plan {
     // runtime state (runtime.cu)
     std::vector<std::shared_ptr<kf::CompiledBlock>> compiled;
     std::map<int, void *> workspace;         // image id -> device buffer (cut edges)
+    std::map<kf::GeomKey, kf::Geom> geom;    // memoised launch geometry (runtime.cu)
     bool prepared = false;
     ~kf_plan();
 };

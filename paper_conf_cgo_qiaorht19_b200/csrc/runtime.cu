@@ -14,6 +14,7 @@
 #include <utime.h>
 #include <unistd.h>
 
+#include <cstddef>
 #include <cstdio>
 #include <cstring>
 #include <fstream>
@@ -426,7 +427,23 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         a.r0 = blo[bi];
         a.r1 = bhi[bi];
         if (a.r1 <= a.r0) continue;
-        unsigned grid = launch_geometry(p, a, b, cb);
+        // The geometry depends only on the block, its output rows and the
+        // run-time schedule options: memoised per plan, so an eager kf_run (and
+        // every band of kf_run_host) skips the strip-count search.
+        const GeomKey gk{(int)bi, a.r0, a.r1, opt(p, "nstrips"), opt(p, "nlong")};
+        unsigned grid;
+        constexpr size_t kTail = offsetof(KfArgs, rect);   // geometry fields: rect[] .. n_long
+        auto git = plan->geom.find(gk);
+        if (git != plan->geom.end()) {
+            std::memcpy((unsigned char *)&a + kTail, git->second.tail.data(), sizeof(KfArgs) - kTail);
+            grid = git->second.grid;
+        } else {
+            grid = launch_geometry(p, a, b, cb);
+            Geom g;
+            g.tail.assign((const unsigned char *)&a + kTail, (const unsigned char *)&a + sizeof(KfArgs));
+            g.grid = grid;
+            plan->geom.emplace(gk, std::move(g));
+        }
         if (!cb.si.ok) a.n_items = 0;   // frame-only block
         {   // Optional persistent CTAs (experimental option "persist"): at most one
             // wave, the kernel strides over the items.  Measured slower (C3 27.4 ->
