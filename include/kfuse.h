@@ -193,7 +193,7 @@ kf_status kf_mark_output(kf_pipeline *p, int32_t image_id);
  * plans prepared afterwards; run-time options (nstrips, host_taper) at the next
  * kf_run.  Names: swar swring swring_cap prefetch sring smem_rows lds_pf
  * const_w pro_rp qptr heavy_first code_budget rolled_edge_v minctas nstrips
- * host_taper host_bands host_direct host_inline_d2h tma rtrip cta_warps peel_warmup.  Unknown names or out-of-range values: KF_ERR_ARG.
+ * host_taper host_bands host_direct tma rtrip cta_warps peel_warmup.  Unknown names or out-of-range values: KF_ERR_ARG.
  * (The measured-and-rejected v8 / persist / persist_waves / nlong and the
  * rounding-changing diagnostics pairs / defer exist only in a KF_EXPERIMENTAL
  * build, and the naive_border negative control only in the KF_TEST_HOOKS build

@@ -2083,7 +2083,6 @@ const OptDef kOpts[] = {
     {"host_taper", 1, 0, 1, false},     // kf_run_host thin first/last bands
     {"host_bands", 8, 1, 32, false},    // kf_run_host row bands (pipeline depth)
     {"host_direct", 0, 0, 1, false},    // kf_run_host: kernels access pinned+mapped host buffers directly
-    {"host_inline_d2h", 0, 0, 1, false},   // kf_run_host: downloads queued on the compute stream
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)

@@ -573,17 +573,11 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
             run(p, plan, din.data(), n_in, dout.data(), n_out, stream, 0, p->H, 0, p->H);
         else
             run(p, plan, din.data(), n_in, dout.data(), n_out, stream, r0, r1, 0, p->H, true);
-        // option host_inline_d2h: the band's download is queued on the compute
-        // stream itself (no cross-stream event), else on the D2H stream
-        const bool inl = opt(p, "host_inline_d2h") != 0;
-        cudaStream_t sd = inl ? s : rt.s_d2h;
-        if (!inl) {
-            KF_CUDA(cudaEventRecord(rt.ev_out[k], s));
-            KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_out[k], 0));
-        }
+        KF_CUDA(cudaEventRecord(rt.ev_out[k], s));
+        KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_out[k], 0));
         for (int j = 0; j < n_out; j++)
             KF_CUDA(cudaMemcpyAsync((char *)hout[j] + r0 * row_bytes, (const char *)rt.stage_out[j] + r0 * row_bytes,
-                                    (r1 - r0) * row_bytes, cudaMemcpyDeviceToHost, sd));
+                                    (r1 - r0) * row_bytes, cudaMemcpyDeviceToHost, rt.s_d2h));
     }
     KF_CUDA(cudaEventRecord(rt.ev_done, rt.s_d2h));
     KF_CUDA(cudaStreamWaitEvent(s, rt.ev_done, 0));

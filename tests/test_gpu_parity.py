@@ -244,7 +244,7 @@ def test_run_host_equals_run(wl, kind, size):
 
 
 @pytest.mark.parametrize("opts", [{"host_bands": 1}, {"host_bands": 3}, {"host_bands": 16}, {"host_bands": 32},
-                                  {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}, {"host_inline_d2h": 1}])
+                                  {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}])
 def test_run_host_pipeline_depth_bit_identical(opts):
     """Any kf_run_host band count / taper (options host_bands, host_taper) gives
     kf_run's bits (each band is a kf_run_band with global border handling)."""

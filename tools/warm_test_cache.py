@@ -91,7 +91,7 @@ def jobs():
         out.append((P.WORKLOADS[wl](300, 200), "b200", None, False))
     out.append((P.harris(512, 384), "b200", None, False))     # examples/harris_c.c
     for o in ({"host_bands": 1}, {"host_bands": 3}, {"host_bands": 16}, {"host_bands": 32},
-              {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}, {"host_inline_d2h": 1}):
+              {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}):
         out.append((P.harris(130, 1030), "b200", o, False))
     return out
 
