@@ -1,4 +1,4 @@
-"""Summarises the ncu DRAM captures of tools/gpu_r1t.sh into a markdown table:
+"""Summarises the ncu DRAM captures (tools/gpu_r2x.sh) into a markdown table:
 measured DRAM bytes per pixel per plan (sum over the plan's launches of one run,
 cold L2: --cache-control all) against the algorithmic bytes of SURVEY §8(d)."""
 import csv
