@@ -8,7 +8,10 @@ terms of O(1), e.g. a zero-sum mask on a 1-pixel-wide image -- is rounding noise
 on both sides and is compared absolutely, <= 1e-6).  Kernels are compiled up
 front in parallel.
 
-    python tests/fuzz_parity.py [n_dags] [seed0]     -> one JSON line, exit 1 on any mismatch
+    python tests/fuzz_parity.py [n_dags] [seed0] [oracle|bands]   -> one JSON line, exit 1 on any mismatch
+
+Mode `bands` checks the decompositions instead: kf_run_host and random row
+bands (kf_run_band) against the whole-image kf_run, bit for bit.
 """
 import json
 import os
@@ -67,12 +70,53 @@ def make(spec, kind, opts, lab):
     return p.plan_fusion(kind)
 
 
+def bands_mode(cases):
+    """Decompositions: every case again as random row bands (kf_run_band from the
+    band's own input rows + halo) and through kf_run_host; both must equal the
+    whole-image kf_run bit for bit (REPEAT plans: run_host only)."""
+    bad = []
+    for spec, kind, opts, lab, seed in cases:
+        H, W = spec["height"], spec["width"]
+        ins = [gen.image(spec["dtype"], seed + 7 * j, W, H) for j in range(spec["n_inputs"])]
+        plan = make(spec, kind, opts, lab)
+        d_in = [torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in ins]
+        shape = (H, W) + (() if spec["dtype"] == "f32" else (4,))
+        dt = torch.float32 if spec["dtype"] == "f32" else torch.uint8
+        full = [torch.empty(shape, dtype=dt, device="cuda") for _ in spec["outputs"]]
+        plan.run(d_in, full)
+        torch.cuda.synchronize()
+        full = [f.cpu().numpy() for f in full]
+        host = [np.empty_like(f) for f in full]
+        plan.run_host([np.ascontiguousarray(a) for a in ins], host)
+        ok = all(np.array_equal(a, b) for a, b in zip(host, full))
+        repeat = any(o["kind"] == "local" and o["mode"] == "repeat" for o in spec["ops"])
+        if ok and not repeat and H >= 2:
+            rng = random.Random(seed)
+            cuts = sorted({0, H} | {rng.randint(1, H - 1) for _ in range(rng.randint(1, 4))})
+            R = plan.halo_rows
+            for r0, r1 in zip(cuts[:-1], cuts[1:]):
+                a0, a1 = max(0, r0 - R), min(H, r1 + R)
+                b_in = [torch.from_numpy(np.ascontiguousarray(x[a0:a1])).cuda() for x in ins]
+                b_out = [torch.empty((r1 - r0,) + shape[1:], dtype=dt, device="cuda") for _ in spec["outputs"]]
+                plan.run_band(r0, r1, b_in, a0, a1, b_out)
+                torch.cuda.synchronize()
+                ok &= all(np.array_equal(o.cpu().numpy(), f[r0:r1]) for o, f in zip(b_out, full))
+        if not ok:
+            bad.append({"seed": seed, "kind": kind, "opts": opts, "size": [W, H], "dtype": spec["dtype"]})
+    return bad
+
+
 def main():
     n = int(sys.argv[1]) if len(sys.argv) > 1 else 200
     seed0 = int(sys.argv[2]) if len(sys.argv) > 2 else 424242
+    mode = sys.argv[3] if len(sys.argv) > 3 else "oracle"
     cases = [case(i, seed0) for i in range(n)]
     with ThreadPoolExecutor(max(1, min(32, os.cpu_count() or 1))) as ex:
         list(ex.map(lambda c: make(*c[:4]).compile(), cases))
+    if mode == "bands":
+        bad = bands_mode(cases)
+        print(json.dumps({"mode": "bands", "dags": n, "seed0": seed0, "mismatches": len(bad), "bad": bad[:20]}))
+        sys.exit(1 if bad else 0)
     bad, worst, cancelled = [], 0.0, []
     for spec, kind, opts, lab, seed in cases:
         ins = [gen.image(spec["dtype"], seed + 7 * j, spec["width"], spec["height"]) for j in range(spec["n_inputs"])]
