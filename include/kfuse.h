@@ -193,7 +193,7 @@ kf_status kf_mark_output(kf_pipeline *p, int32_t image_id);
  * plans prepared afterwards; run-time options (nstrips, host_taper) at the next
  * kf_run.  Names: swar swring swring_cap prefetch sring smem_rows lds_pf
  * const_w pro_rp qptr heavy_first code_budget rolled_edge_v minctas nstrips
- * host_taper host_bands host_direct tma rtrip cta_warps peel_warmup.  Unknown names or out-of-range values: KF_ERR_ARG.
+ * host_taper host_bands host_direct tma rtrip cta_warps peel_warmup pdl.  Unknown names or out-of-range values: KF_ERR_ARG.
  * (The measured-and-rejected v8 / persist / persist_waves / nlong and the
  * rounding-changing diagnostics pairs / defer exist only in a KF_EXPERIMENTAL
  * build, and the naive_border negative control only in the KF_TEST_HOOKS build
@@ -268,6 +268,22 @@ kf_status kf_compile_plan(kf_pipeline *p, const kf_plan *plan);
  * on `stream`, in topological block order.  No allocation after kf_prepare. */
 kf_status kf_run(kf_pipeline *p, const kf_plan *plan, const void *const *d_inputs, int32_t n_in,
                  void *const *d_outputs, int32_t n_out, void *stream);
+
+/* A batch of INDEPENDENT frames (e.g. consecutive video frames): frame f reads
+ * d_inputs[f*n_in + i] and writes d_outputs[f*n_out + j], with kf_run's layout,
+ * alignment and result for every frame (bit-identical to n_frames kf_run
+ * calls).  Every output image must be disjoint from every other frame's input
+ * and output images (inputs may be shared), else KF_ERR_ARG before any launch.
+ * Single-block plans launch frames 1..n-1 as programmatic dependent launches
+ * that do not wait for the previous frame (only for its completion at their
+ * end): the next frame's CTAs fill the SM slots the previous frame's tail
+ * leaves idle.  Frame 0 waits for all earlier work on `stream` as kf_run does,
+ * and completion of the last frame implies completion of all of them.
+ * Multi-block plans share one workspace and run the frames in order.
+ * Same paper passage as kf_run (one kernel per block); the
+ * frame overlap is a B200 scheduling choice. */
+kf_status kf_run_batch(kf_pipeline *p, const kf_plan *plan, int32_t n_frames, const void *const *d_inputs,
+                       int32_t n_in, void *const *d_outputs, int32_t n_out, void *stream);
 
 /* End-to-end call with HOST buffers: copies inputs host->device, runs, copies
  * outputs device->host, synchronises `stream`.  The image is processed in up to

@@ -350,6 +350,15 @@ kf_status kf_run(kf_pipeline *p, const kf_plan *plan, const void *const *d_input
     });
 }
 
+kf_status kf_run_batch(kf_pipeline *p, const kf_plan *plan, int32_t n_frames, const void *const *d_inputs,
+                       int32_t n_in, void *const *d_outputs, int32_t n_out, void *stream)
+{
+    return guard([&] {
+        if (!p || !plan || plan->pipe != p) fail(KF_ERR_ARG, "plan does not belong to pipeline");
+        run_batch(p, const_cast<kf_plan *>(plan), n_frames, d_inputs, n_in, d_outputs, n_out, stream);
+    });
+}
+
 kf_status kf_run_host(kf_pipeline *p, const kf_plan *plan, const void *const *h_inputs, int32_t n_in,
                       void *const *h_outputs, int32_t n_out, void *stream)
 {

@@ -959,6 +959,7 @@ struct StreamGen {
     bool qptr = false;     // steady-state loop: ring slots addressed from per-trip base pointers
     bool tma = false;      // this variant feeds the ring with TMA bulk row copies (option tma)
     int peel_Q = 0;        // peeled iterations of the variant being emitted
+    int loop_u0 = 0;       // first iteration of the steady-state loop of the variant being emitted
 
     StreamGen(const kf_pipeline *p_, const BlockInfo &b_, const StreamInfo &si_, int block_, std::ostringstream &o_)
         : p(p_), b(b_), si(si_), block(block_), f32(p_->dtype == KF_F32), o(o_), pe{p_->dtype == KF_F32, block_, &tmp},
@@ -1653,10 +1654,41 @@ struct StreamGen {
         } else {
             for (int img : b.ext) load(img, sl(img, D, j), uexpr + " + " + std::to_string(j + D), ind);
         }
+        // Kernel k is first needed at iteration 2L - 2 HY(k): its row then is the
+        // first of the rows [ys - HY(k), ye + HY(k)) the strip's outputs read.
+        // A peeled iteration skips it statically.  In the loop (option
+        // warm_skip), kernels first needed after the loop's first iteration run
+        // under a warp-uniform guard, so the warm-up rows of a loop that starts
+        // at iteration 0 (rolled bodies) compute only what later rows read.
+        // Consumers never read a skipped row (HY(producer) >= HY(consumer) +
+        // ry(consumer)).  Temporaries of a guarded group go out of scope with it,
+        // so the value memos are cleared after each group.  An int32 (I4) sink
+        // whose ring is not written is stored from its memoised temporaries,
+        // so it stays unguarded.
+        const bool i4_sink_memo = !f32 && !si.swk.count(b.sink) && si.depth.at(p->n_inputs + b.sink) <= 1;
+        int group = -1;
         for (int k : b.kernels) {
-            // warm-up (peeled) iteration: kernel k is first needed at iteration 2L - 2 HY(k)
-            if (u >= 0 && u < 2 * L - 2 * HY(p->n_inputs + k)) continue;
-            kernel(k, j, u, ind);
+            const int first = 2 * L - 2 * HY(p->n_inputs + k);
+            if (u >= 0) {
+                if (u < first) continue;
+                kernel(k, j, u, ind);
+                continue;
+            }
+            const bool guard = opt(p, "warm_skip") && first > loop_u0 + j && !(k == b.sink && i4_sink_memo);
+            const int g = guard ? first : -1;
+            if (g != group) {
+                if (group >= 0) {
+                    o << ind << "}\n";
+                    val_memo.clear(); shfl_memo.clear(); sw_memo.clear(); swsh_memo.clear();
+                }
+                if (g >= 0) o << ind << "if (" << uexpr << " + " << j << " >= " << first << ") {\n";
+                group = g;
+            }
+            kernel(k, j, u, group >= 0 ? ind + "    " : ind);
+        }
+        if (group >= 0) {
+            o << ind << "}\n";
+            val_memo.clear(); shfl_memo.clear(); sw_memo.clear(); swsh_memo.clear();
         }
         const int simg = p->n_inputs + b.sink;
         const int ss = sl(simg, 0, j);
@@ -1907,6 +1939,7 @@ struct StreamGen {
             o << "    " << RT() << " *__restrict__ op = gout + " << (dir > 0 ? yp0 : "(H - 1 - " + yp0 + ")") << " * W;\n";
             runptr = true;
         }
+        loop_u0 = u0;
         if (si.rolled) {
             const int T = si.T;
             o << "    #pragma unroll 1\n";
@@ -2085,6 +2118,9 @@ const OptDef kOpts[] = {
     {"host_direct", 0, 0, 1, false},    // kf_run_host: kernels access pinned+mapped host buffers directly
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)
+    {"warm_skip", 1, 0, 1, false},      // loop warm-up rows skip kernels not yet needed (rolled bodies)
+    {"pdl", 0, 0, 1, false},            // kf_run kernels launched as programmatic dependents (the CTA
+                                        // launch overlaps the previous kernel's tail; measured mixed, off)
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
     {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
     {"persist_waves", 1, 1, 1 << 20, true},
@@ -2342,6 +2378,18 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     // items (every issued row was waited for), so the shared ring is reused.
     // With NW > 1 warps per CTA a frame unit uses all of them (its loops stride
     // by blockDim), an interior unit gives each warp its own item and ring.
+    // Programmatic dependent launch.  Without the launch
+    // attribute both instructions are no-ops.  With it: a dependent kernel
+    // (indep = 0: kf_run, the first frame of kf_run_batch, every block of a
+    // multi-block plan) waits for the previous grid -- its completion and the
+    // visibility of its writes -- before the first global access, then lets
+    // the next kernel be scheduled.  An independent frame (indep = 1: frames
+    // after the first of kf_run_batch, whose buffers the runtime checked to be
+    // disjoint) lets the next kernel be scheduled at once and waits for the
+    // previous grid only at its end, so its completion still implies the
+    // completion of every earlier kernel on the stream.
+    o << "    if (!a.indep) asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n";
+    o << "    asm volatile(\"griddepcontrol.launch_dependents;\");\n";
     o << "    const int total = a.frame_ctas + (a.n_items + " << NW - 1 << ") / " << NW << ";\n";
     o << "    for (int cta = blockIdx.x; cta < total; cta += gridDim.x) {\n";
     o << "        if (cta < a.frame_ctas) " << kernel_name(block) << "_frame(a, cta);\n";
@@ -2357,6 +2405,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     }
     o << (NW == 1 ? "        __syncwarp();\n" : "        __syncthreads();\n");
     o << "    }\n";
+    o << "    if (a.indep) asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n";
     o << "}\n";
     return o.str();
 }

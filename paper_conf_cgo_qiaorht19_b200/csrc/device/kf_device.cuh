@@ -29,6 +29,8 @@ struct KfArgs {
     int out_base;                  // global row held by row 0 of `out`
     int W, H;                      // image size (global)
     int r0, r1;                    // output rows computed by this launch
+    int indep;                     // 1: independent of the previous kernel on the stream (kf_run_batch
+                                   // frames after the first): griddepcontrol.wait moves to the kernel's end
     // border frame: slow path, CTAs [0, frame_ctas)
     KfRect rect[KF_MAX_RECT];
     int n_rect, frame_ctas;

@@ -184,7 +184,10 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block);
 // runtime.cu
 void prepare(kf_pipeline *p, kf_plan *plan);
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
-         void *stream, int row0, int row1, int in_row0, int in_row1, bool out_full = false);
+         void *stream, int row0, int row1, int in_row0, int in_row1, bool out_full = false,
+         bool indep = false);
+void run_batch(kf_pipeline *p, kf_plan *plan, int n_frames, const void *const *din, int n_in,
+               void *const *dout, int n_out, void *stream);
 void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
               void *stream);
 void release_plan(kf_plan *plan);

@@ -14,6 +14,7 @@
 #include <utime.h>
 #include <unistd.h>
 
+#include <algorithm>
 #include <cstddef>
 #include <cstdio>
 #include <cstring>
@@ -52,6 +53,7 @@ struct Driver {
     CUresult (*moduleUnload)(CUmodule) = nullptr;
     CUresult (*launchKernel)(CUfunction, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned, unsigned,
                              CUstream, void **, void **) = nullptr;
+    CUresult (*launchKernelEx)(const CUlaunchConfig *, CUfunction, void **, void **) = nullptr;
     CUresult (*getErrorString)(CUresult, const char **) = nullptr;
     CUresult (*occupancy)(int *, CUfunction, int, size_t) = nullptr;
 };
@@ -79,6 +81,7 @@ static Driver &driver()
         get("cuModuleGetFunction", (void **)&d.moduleGetFunction);
         get("cuModuleUnload", (void **)&d.moduleUnload);
         get("cuLaunchKernel", (void **)&d.launchKernel);
+        get("cuLaunchKernelEx", (void **)&d.launchKernelEx);
         get("cuGetErrorString", (void **)&d.getErrorString);
         get("cuOccupancyMaxActiveBlocksPerMultiprocessor", (void **)&d.occupancy);
     });
@@ -351,7 +354,7 @@ static unsigned launch_geometry(const kf_pipeline *p, KfArgs &a, const BlockInfo
 }
 
 void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *const *dout, int n_out,
-         void *stream, int row0, int row1, int in_row0, int in_row1, bool out_full)
+         void *stream, int row0, int row1, int in_row0, int in_row1, bool out_full, bool indep)
 {
     if (n_in != p->n_inputs || (n_in && !din)) fail(KF_ERR_ARG, "wrong number of inputs");
     if (n_out != (int)p->outputs.size() || (n_out && !dout)) fail(KF_ERR_ARG, "wrong number of outputs");
@@ -426,6 +429,7 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         a.H = p->H;
         a.r0 = blo[bi];
         a.r1 = bhi[bi];
+        a.indep = indep ? 1 : 0;
         if (a.r1 <= a.r0) continue;
         // The geometry depends only on the block, its output rows and the
         // run-time schedule options: memoised per plan, so an eager kf_run (and
@@ -455,7 +459,32 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         }
         if (grid == 0) continue;
         void *params[] = {&a};
-        cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads * cb.si.nw, 1, 1, 0, st, params, nullptr), "cuLaunchKernel");
+        if (indep || opt(p, "pdl")) {
+            // Programmatic dependent launch: this grid may be
+            // scheduled once every CTA of the previous kernel on the stream has
+            // triggered (this library's kernels trigger after their own wait).
+            // A dependent kernel (indep = 0) executes griddepcontrol.wait before
+            // its first global access: stream order is kept and only the CTA
+            // launch overlaps the previous tail.  An independent frame of
+            // kf_run_batch runs concurrently with the previous frame's tail and
+            // waits for it at its end.
+            CUlaunchAttribute attr[1];
+            std::memset(attr, 0, sizeof attr);
+            attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+            attr[0].value.programmaticStreamSerializationAllowed = 1;
+            CUlaunchConfig cfg;
+            std::memset(&cfg, 0, sizeof cfg);
+            cfg.gridDimX = grid; cfg.gridDimY = 1; cfg.gridDimZ = 1;
+            cfg.blockDimX = kThreads * cb.si.nw; cfg.blockDimY = 1; cfg.blockDimZ = 1;
+            cfg.sharedMemBytes = 0;
+            cfg.hStream = st;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            cu_check(d.launchKernelEx(&cfg, cb.fn, params, nullptr), "cuLaunchKernelEx");
+        } else {
+            cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads * cb.si.nw, 1, 1, 0, st, params, nullptr),
+                     "cuLaunchKernel");
+        }
     }
     for (auto &c : band_copies) {
         const char *src = (const char *)plan->workspace[c.first] + (size_t)row0 * p->W * 4;
@@ -463,6 +492,41 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         KF_CUDA(cudaMemcpyAsync(dst, src, (size_t)(row1 - row0) * p->W * 4, cudaMemcpyDeviceToDevice,
                                 (cudaStream_t)stream));
     }
+}
+
+// Independent frames (kf_run_batch): frame f runs the plan on
+// din[f*n_in ..], dout[f*n_out ..].  Single-block plans launch the frames
+// after the first as programmatic dependents that need not wait (indep): the
+// CTAs of frame f+1 fill the SM slots that frame f's tail leaves idle.  That is
+// only correct when no frame writes memory another frame touches, so every
+// output image is checked to be disjoint from every other frame's images.
+// Multi-block plans share one workspace between frames and run them in order.
+void run_batch(kf_pipeline *p, kf_plan *plan, int n_frames, const void *const *din, int n_in,
+               void *const *dout, int n_out, void *stream)
+{
+    if (n_frames < 0) fail(KF_ERR_ARG, "negative frame count");
+    if (n_frames == 0) return;
+    if (n_in != p->n_inputs || n_out != (int)p->outputs.size()) fail(KF_ERR_ARG, "wrong number of buffers");
+    if ((n_in && !din) || (n_out && !dout)) fail(KF_ERR_ARG, "null buffer array");
+    const uintptr_t bytes = (uintptr_t)p->W * p->H * 4;
+    struct Span { uintptr_t lo, hi; int frame; bool out; };
+    std::vector<Span> spans;
+    for (int f = 0; f < n_frames; f++) {
+        for (int i = 0; i < n_in; i++) spans.push_back({(uintptr_t)din[f * n_in + i], (uintptr_t)din[f * n_in + i] + bytes, f, false});
+        for (int j = 0; j < n_out; j++) spans.push_back({(uintptr_t)dout[f * n_out + j], (uintptr_t)dout[f * n_out + j] + bytes, f, true});
+    }
+    std::sort(spans.begin(), spans.end(), [](const Span &x, const Span &y) { return x.lo < y.lo; });
+    // any overlap of two spans of different frames, one of them written, is a hazard
+    for (size_t i = 0; i < spans.size(); i++)
+        for (size_t j = i + 1; j < spans.size() && spans[j].lo < spans[i].hi; j++)
+            if (spans[i].frame != spans[j].frame && (spans[i].out || spans[j].out))
+                fail(KF_ERR_ARG, "kf_run_batch: frames " + std::to_string(spans[i].frame) + " and " +
+                                     std::to_string(spans[j].frame) + " share memory that one of them writes");
+    prepare(p, plan);
+    const bool overlap = plan->blocks.size() == 1;
+    for (int f = 0; f < n_frames; f++)
+        run(p, plan, din + (size_t)f * n_in, n_in, dout + (size_t)f * n_out, n_out, stream, 0, p->H, 0, p->H,
+            false, overlap && f > 0);
 }
 
 // End-to-end call with host buffers.  The image is cut into kHostBands row

@@ -87,6 +87,7 @@ _SIGS = {
     "kf_prepare": (C.c_int, [_P, _P]),
     "kf_run": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_host": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
+    "kf_run_batch": (C.c_int, [_P, _P, C.c_int32, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_band": (C.c_int, [_P, _P, C.c_int32, C.c_int32, C.POINTER(_P), C.c_int32, C.c_int32,
                               C.POINTER(_P), _P]),
     "kf_set_option": (C.c_int, [_P, C.c_char_p, C.c_int64]),
@@ -324,6 +325,20 @@ class Plan:
         stream: a torch.cuda.Stream, a raw cudaStream_t int, or None = torch's current stream."""
         _check(lib.kf_run(self.pipe.h, self.h, _ptrs([_dptr(t) for t in inputs]), len(inputs),
                           _ptrs([_dptr(t) for t in outputs]), len(outputs), _P(_stream(stream))))
+
+    def run_batch(self, frames_in, frames_out, stream=None) -> None:
+        """Independent frames (kf_run_batch): frames_in[f] / frames_out[f] are the
+        input / output lists of frame f, as for run()."""
+        n = len(frames_in)
+        if len(frames_out) != n:
+            raise ValueError("frames_in and frames_out differ in length")
+        n_in = len(frames_in[0]) if n else self.pipe.n_inputs
+        n_out = len(frames_out[0]) if n else 0
+        if any(len(f) != n_in for f in frames_in) or any(len(f) != n_out for f in frames_out):
+            raise ValueError("every frame needs the same number of inputs and outputs")
+        _check(lib.kf_run_batch(self.pipe.h, self.h, n,
+                                _ptrs([_dptr(t) for f in frames_in for t in f]), n_in,
+                                _ptrs([_dptr(t) for f in frames_out for t in f]), n_out, _P(_stream(stream))))
 
     def run_host(self, inputs, outputs, stream=None) -> None:
         """End-to-end: host numpy/pinned-tensor buffers in and out (kf_run_host)."""

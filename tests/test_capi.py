@@ -126,6 +126,25 @@ def test_argument_validation():
         K.Pipeline(0, 5, "f32")
 
 
+def test_run_batch_validates_frames_without_a_gpu():
+    """kf_run_batch checks frame disjointness before touching CUDA: an output that
+    overlaps another frame's input or output is KF_ERR_ARG; so is a negative count;
+    zero frames is a no-op.  (Addresses are never dereferenced on this path.)"""
+    spec = P.harris(64, 32)
+    plan = K.Pipeline.from_spec(spec).plan_fusion("b200")
+    nb = 64 * 32 * 4
+    base = 1 << 40
+    with pytest.raises(K.KfError) as e:      # frame 1 reads frame 0's output
+        plan.run_batch([[base], [base + nb]], [[base + nb], [base + 2 * nb]], stream=0)
+    assert e.value.name == "KF_ERR_ARG" and "share memory" in str(e.value)
+    with pytest.raises(K.KfError) as e:      # outputs overlap by one pixel
+        plan.run_batch([[base], [base]], [[base + nb], [base + 2 * nb - 4]], stream=0)
+    assert e.value.name == "KF_ERR_ARG"
+    plan.run_batch([], [], stream=0)
+    st = K.lib.kf_run_batch(plan.pipe.h, plan.h, -1, K._ptrs([base]), 1, K._ptrs([base + nb]), 1, None)
+    assert st != 0
+
+
 def test_peer_calls_validate_without_a_gpu():
     """The multi-GPU entry points check their arguments before touching CUDA:
     same-device peer enable is a no-op; bad segment counts fail with KF_ERR_ARG."""

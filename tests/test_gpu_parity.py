@@ -260,6 +260,77 @@ def test_run_host_pipeline_depth_bit_identical(opts):
     np.testing.assert_array_equal(hout.numpy(), dev)
 
 
+@pytest.mark.parametrize("wl,kind,size", [("harris", "b200", (300, 200)), ("harris", "b200", (1024, 768)),
+                                          ("deep10", "b200", (260, 150)), ("unsharp", "b200", (2048, 512)),
+                                          ("two_input", "b200", (512, 300)), ("harris", "unfused", (300, 200)),
+                                          ("harris", "paper", (256, 256))])
+def test_run_batch_equals_run(wl, kind, size):
+    """kf_run_batch (frames after the first overlap the previous frame's tail through
+    programmatic dependent launch) == one kf_run per frame, bit for bit -- with the
+    inputs written by torch kernels just before the batch on the same stream (frame
+    0 must wait for them, and frames 1.. may only start once frame 0 has) and the
+    outputs read by torch kernels right after it (the last frame's completion must
+    imply every frame's)."""
+    spec = P.WORKLOADS[wl](*size)
+    nf = 6
+    frames = [_inputs(spec, 40 + f) for f in range(nf)]
+    plan = make_plan(spec, kind)
+    refs = [run_gpu(spec, plan, ins) for ins in frames]
+    src = [[torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in ins] for ins in frames]
+    d_in = [[torch.zeros_like(t) for t in f] for f in src]
+    outs = [_alloc(spec) for _ in range(nf)]
+    for o in outs:
+        for t in o:
+            t.fill_(7)
+    torch.cuda.synchronize()
+    st = torch.cuda.Stream()
+    with torch.cuda.stream(st):
+        for f in range(nf):
+            for t, s in zip(d_in[f], src[f]):
+                t.copy_(s)
+        plan.run_batch(d_in, outs, st)
+        got = [[t.clone() for t in o] for o in outs]
+    torch.cuda.synchronize()
+    for f in range(nf):
+        for g, r in zip(got[f], refs[f]):
+            np.testing.assert_array_equal(g.cpu().numpy(), r, err_msg=f"frame {f}")
+    # graph-captured batch replay, a shared input, a plain kf_run chained after it
+    shared = [[src[0][0]] + f[1:] for f in d_in]
+    for o in outs:
+        for t in o:
+            t.fill_(3)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=st):
+        plan.run_batch(shared, outs, st)
+    with torch.cuda.stream(st):
+        g.replay()
+        chained = _alloc(spec)
+        plan.run(d_in[-1], chained, st)
+        tail = [t.clone() for t in outs[-1]]
+    torch.cuda.synchronize()
+    ref_shared = [run_gpu(spec, plan, [frames[0][0]] + frames[f][1:]) for f in range(nf)]
+    for f in range(nf):
+        for t, r in zip(outs[f], ref_shared[f]):
+            np.testing.assert_array_equal(t.cpu().numpy(), r, err_msg=f"graph frame {f}")
+    np.testing.assert_array_equal(tail[0].cpu().numpy(), ref_shared[-1][0])
+    np.testing.assert_array_equal(chained[0].cpu().numpy(), refs[-1][0])
+
+
+def test_run_batch_rejects_shared_outputs():
+    """A frame writing memory another frame reads or writes is rejected before any launch."""
+    spec = P.harris(128, 64)
+    plan = make_plan(spec, "b200")
+    a, b = (torch.zeros(64, 128, device="cuda") for _ in range(2))
+    big = torch.zeros(2 * 64, 128, device="cuda")
+    with pytest.raises(K.KfError):
+        plan.run_batch([[a], [b]], [[b], [big[:64]]])          # frame 1 reads frame 0's output
+    with pytest.raises(K.KfError):
+        plan.run_batch([[a], [a]], [[big[:64]], [big[32:96]]])  # overlapping outputs
+    plan.run_batch([[a], [a]], [[big[:64]], [big[64:]]])        # shared input, disjoint outputs: fine
+    plan.run_batch([], [])
+    torch.cuda.synchronize()
+
+
 def test_run_host_repeat_and_pinned():
     """REPEAT plans (one band) and pinned host buffers on a non-default stream."""
     spec = P.harris(256, 300, "repeat")
@@ -551,7 +622,7 @@ SAME_BITS = [{"qptr": 0}, {"lds_pf": 0}, {"const_w": 0}, {"heavy_first": 0}, {"p
              {"tma": 1, "lds_pf": 0}, {"tma": 1, "code_budget": 1000}, {"tma": 1, "smem_rows": 6}, {"rtrip": 2},
              {"rtrip": 2, "code_budget": 1000}, {"code_budget": 1000, "lds_pf": 0}, {"cta_warps": 2},
              {"cta_warps": 4}, {"cta_warps": 8}, {"cta_warps": 4, "tma": 1}, {"cta_warps": 4, "code_budget": 1000},
-             {"peel_warmup": 0}, {"peel_warmup": 0, "lds_pf": 0}]
+             {"peel_warmup": 0}, {"peel_warmup": 0, "lds_pf": 0}, {"pdl": 0}]
 EXPERIMENTAL = [{"v8": 1}, {"persist": 1}, {"nlong": 3}, {"persist": 1, "persist_waves": 2}]
 # experimental options that change the f32 rounding (scalar instead of packed pairs,
 # scales applied per stage): within the parity tolerance of the oracle, not bit-identical

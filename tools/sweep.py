@@ -15,11 +15,25 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
-def time_setting(cfg: str, plan_kind: str, steps: int, opts: dict, reps: int) -> dict:
+def _binding(lib: str):
+    """The product binding, or a second instance bound to the test-hooks build
+    (experimental options) when lib == 'testhooks'."""
+    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+    if lib != "testhooks":
+        return K
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("kfuse_testhooks", K.__file__)
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    mod.lib = mod._open(os.path.join(os.path.dirname(K.__file__), "libkfuse_testhooks.so"))
+    return mod
+
+
+def time_setting(cfg: str, plan_kind: str, steps: int, opts: dict, reps: int, lib: str = "product") -> dict:
     import torch
     from kf_inputs import gen
     from kf_inputs import pipelines as P
-    from paper_conf_cgo_qiaorht19_b200 import kfuse as K
+    K = _binding(lib)
     if ":" in cfg:   # workload:W:H
         wl, w, h = cfg.split(":")
         spec, seed = P.WORKLOADS[wl](int(w), int(h)), 1
@@ -67,6 +81,7 @@ def main():
     ap.add_argument("--plan", default="b200")
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--reps", type=int, default=7)
+    ap.add_argument("--lib", default="product", choices=["product", "testhooks"])
     ap.add_argument("settings", nargs="*")
     a = ap.parse_args()
     for st in a.settings or [""]:
@@ -75,10 +90,10 @@ def main():
             k, v = kv.split("=", 1)
             opts[k] = int(v)
         try:
-            r = time_setting(a.config, a.plan, a.steps, opts, a.reps)
+            r = time_setting(a.config, a.plan, a.steps, opts, a.reps, a.lib)
         except Exception as e:   # noqa: BLE001
             r = {"error": f"{type(e).__name__}: {str(e)[:300]}"}
-        print(json.dumps({"config": a.config, "plan": a.plan, "setting": st, **r}), flush=True)
+        print(json.dumps({"config": a.config, "plan": a.plan, "lib": a.lib, "setting": st, **r}), flush=True)
 
 
 if __name__ == "__main__":
