@@ -290,7 +290,7 @@ def time_batch(plan, ins, outs, frames, steps, stream, torch):
     return t0.elapsed_time(t1) / (nb * frames)
 
 
-def frames_block(plan, host, oshape, tdt, px, ab, single_ms, steps, stream, torch) -> dict:
+def frames_block(plan, host, oshape, tdt, px, ab, single_ms, steps, stream, torch, what=True) -> dict:
     """A stream of independent frames of the workload through kf_run_batch
     (frames after the first overlap the previous frame's tail):
     ms per frame, Mpixel/s and HBM fraction, beside the single-image kf_run."""
@@ -300,12 +300,14 @@ def frames_block(plan, host, oshape, tdt, px, ab, single_ms, steps, stream, torc
     del ins, outs
     torch.cuda.empty_cache()
     peak = load_peaks()["hbm_gbs"]
-    return {"frames_per_call": FRAMES, "ms_per_frame": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
-            "hbm_frac": round(ab * px / (ms * 1e-3) / 1e9 / peak, 4),
-            "vs_single_kf_run": round(single_ms / ms, 3),
-            "what": "kf_run_batch over independent frames (disjoint buffers): frame f+1's CTAs fill the SM "
-                    "slots frame f's tail leaves idle (programmatic dependent launch); not the headline, "
-                    "which is one kf_run per image"}
+    d = {"frames_per_call": FRAMES, "ms_per_frame": round(ms, 5), "mpix_s": round(px / (ms * 1e-3) / 1e6, 1),
+         "hbm_frac": round(ab * px / (ms * 1e-3) / 1e9 / peak, 4),
+         "vs_single_kf_run": round(single_ms / ms, 3)}
+    if what:
+        d["what"] = ("kf_run_batch over independent frames (disjoint buffers): frame f+1's CTAs fill the SM "
+                     "slots frame f's tail leaves idle (programmatic dependent launch); not the headline, "
+                     "which is one kf_run per image")
+    return d
 
 
 def bench_single(args, cfg_name, spec, seed) -> None:
@@ -512,7 +514,7 @@ def bench_extra(args, stream, torch, clocks) -> dict:
             torch.cuda.empty_cache()
             steps = 16 if px > 1e8 else 40 if px > 2e7 else 200
             d["frames"] = frames_block(fplan, host, oshape, tdt, px, alg_bytes_per_px(spec, fplan.blocks),
-                                       f["ms_per_step"], steps, stream, torch)
+                                       f["ms_per_step"], steps, stream, torch, what=False)
             ins, outs = [], []
         ipp = ncu_inst(cfg, "b200")
         if ipp:
