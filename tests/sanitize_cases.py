@@ -1,8 +1,8 @@
 """TEST INFRASTRUCTURE (not collected by pytest): small launches of every kernel
 family for compute-sanitizer (tools/sanitize.sh):
 C1 Harris 256^2 under every plan, deep10 67x41, all five border modes fused
-(Harris and deep10), 10 random DAGs (3 plans each), the TMA row feed, kf_run_host
-and a row band.  Each result is also checked against the oracle, so a run under
+(Harris and deep10), 10 random DAGs (3 plans each), the TMA row feed, kf_run_host,
+a row band and kf_run_batch frames.  Each result is also checked against the oracle, so a run under
 the sanitizer is a parity run too.  Exit code 0 = all outputs correct."""
 import os
 import random
@@ -71,6 +71,17 @@ def main():
         torch.cuda.synchronize()
         assert torch.equal(band, outs[0][50:110])
         n += 2
+        # kf_run_batch: frames overlapping through programmatic dependent launch
+        for spec, kind in ((P.harris(300, 200), "b200"), (P.deep10(67, 41), "b200"), (P.harris(64, 48), "unfused")):
+            plan, ins, outs = run(spec, kind)
+            shape, dt = outs[0].shape, outs[0].dtype
+            fin = [[torch.from_numpy(np.ascontiguousarray(ins[0])).cuda()] for _ in range(3)]
+            fout = [[torch.empty(shape, dtype=dt, device="cuda")] for _ in range(3)]
+            plan.run_batch(fin, fout)
+            torch.cuda.synchronize()
+            for f in fout:
+                assert torch.equal(f[0], outs[0]), spec["name"]
+            n += 1
     if which in ("all", "random"):
         for seed in range(10):
             rng = random.Random(70000 + seed)
