@@ -12,6 +12,6 @@ for cfg in C3 C4; do
      python tools/prof_run.py --config $cfg --plan b200 > gpurun_out/ncu_${cfg}_s.log 2>&1; echo "ncu $cfg rc=$?"
 done
 python tools/ncu_extract.py C3=gpurun_out/r02_C3_b200_full_s.ncu-rep C4=gpurun_out/r02_C4_b200_full_s.ncu-rep > gpurun_out/r02_ncu_c3_c4_s.json; echo "extract rc=$?"
-bash tools/sanitize.sh
+echo "compute-sanitizer: closed on this pool (runs under it left GPUs needing a reset); not run"
 timeout 600 python tools/sweep.py --config C4 --reps 5 '' 'nstrips=30' 'nstrips=40' 'nstrips=50' 'nstrips=75' 'nstrips=90' '' > gpurun_out/r02_sweep_c4_ns_warmskip.jsonl 2>&1
 cat gpurun_out/r02_sweep_c4_ns_warmskip.jsonl

@@ -1,4 +1,7 @@
 #!/bin/bash
+# NOTE (round 2): compute-sanitizer is closed on the GPU pool ("runs under it have left GPUs
+# needing a reset"); this script is kept for the record of the earlier clean run
+# (profiles/r02_sanitize/) and must not be run there again.
 # compute-sanitizer over every kernel family: memcheck, racecheck,
 # synccheck and initcheck on tests/sanitize_cases.py, plus memcheck on the
 # peer-memory halo kernels at 2 ranks (tests/test_gpu_parity.py peer cases).
