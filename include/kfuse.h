@@ -285,6 +285,16 @@ kf_status kf_run(kf_pipeline *p, const kf_plan *plan, const void *const *d_input
 kf_status kf_run_batch(kf_pipeline *p, const kf_plan *plan, int32_t n_frames, const void *const *d_inputs,
                        int32_t n_in, void *const *d_outputs, int32_t n_out, void *stream);
 
+/* Bounds-checking build (libkfuse_bounds.so, built from the same sources with
+ * KF_BOUNDS; tests only): every global read of a generated kernel must fall
+ * inside one of the launch's external image buffers and every write inside the
+ * launch's own output rows; an access outside is skipped and counted instead of
+ * faulting.  Returns, and clears, the pipeline's record: the
+ * number of violations since the last call, the first offending address and
+ * its kind (0 read, 1 write, 2 table index; the index is then in the low 32
+ * bits).  Synchronises the device.  Every other build: KF_ERR_ARG. */
+kf_status kf_bounds_report(kf_pipeline *p, int64_t *violations, uint64_t *first_addr, int32_t *first_kind);
+
 /* End-to-end call with HOST buffers: copies inputs host->device, runs, copies
  * outputs device->host, synchronises `stream`.  The image is processed in up to
  * 8 row bands on three engines: the H2D copy of band k+1's input rows, the

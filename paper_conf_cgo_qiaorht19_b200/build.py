@@ -51,6 +51,7 @@ def _digest(paths) -> str:
 VARIANTS = {
     "libkfuse.so": [],
     "libkfuse_testhooks.so": ["-DKF_TEST_HOOKS", "-DKF_EXPERIMENTAL"],
+    "libkfuse_bounds.so": ["-DKF_BOUNDS"],
 }
 
 

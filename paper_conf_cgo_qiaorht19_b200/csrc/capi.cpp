@@ -359,6 +359,20 @@ kf_status kf_run_batch(kf_pipeline *p, const kf_plan *plan, int32_t n_frames, co
     });
 }
 
+kf_status kf_bounds_report(kf_pipeline *p, int64_t *violations, uint64_t *first_addr, int32_t *first_kind)
+{
+    return guard([&] {
+        if (!p || !violations || !first_addr || !first_kind) fail(KF_ERR_ARG, "null argument");
+        long long c = 0;
+        unsigned long long ad = 0;
+        int k = 0;
+        bounds_report(p, &c, &ad, &k);
+        *violations = c;
+        *first_addr = ad;
+        *first_kind = k;
+    });
+}
+
 kf_status kf_run_host(kf_pipeline *p, const kf_plan *plan, const void *const *h_inputs, int32_t n_in,
                       void *const *h_outputs, int32_t n_out, void *stream)
 {
@@ -406,8 +420,10 @@ kf_status kf_get_option(const kf_pipeline *p, const char *name, int64_t *value)
 
 const char *kf_version(void)
 {
-#ifdef KF_TEST_HOOKS
+#if defined(KF_TEST_HOOKS)
     return "kfuse 0.2 (sm_100a) TEST HOOKS BUILD -- negative controls, not the product library";
+#elif defined(KF_BOUNDS)
+    return "kfuse 0.2 (sm_100a) BOUNDS-CHECKING BUILD -- checked global accesses, not the product library";
 #else
     return "kfuse 0.2 (sm_100a)";
 #endif

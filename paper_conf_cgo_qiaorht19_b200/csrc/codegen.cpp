@@ -550,8 +550,8 @@ struct SwEmitter {
             for (int c = 0; c < 4; c++) {
                 t[c] = var();
                 const std::string &w = c < 2 ? x.lo : x.hi;
-                *o << ind << "const unsigned " << t[c] << " = (unsigned)__ldg(" << lut_sym << " + "
-                   << (c % 2 ? "(" + w + " >> 16)" : "(" + w + " & 0xffffu)") << ");\n";
+                *o << ind << "const unsigned " << t[c] << " = (unsigned)__ldg(" << lut_sym << " + KF_IDX("
+                   << (c % 2 ? "(" + w + " >> 16)" : "(" + w + " & 0xffffu)") << ", " << n << "));\n";
             }
             r.lo = var();
             r.hi = var();
@@ -1505,16 +1505,16 @@ struct StreamGen {
             unpack_row(img, rs, q, ind);
         } else if (pm) {
             for (int q = 0; q < V / 2; q++)
-                o << ind << ring(img, rs, q) << " = make_float2(__ldg(" << ptr << " + cl" << 2 * q << "), __ldg(" << ptr
+                o << ind << ring(img, rs, q) << " = make_float2(KF_LDG(" << ptr << " + cl" << 2 * q << "), KF_LDG(" << ptr
                   << " + cl" << 2 * q + 1 << "));\n";
         } else if (si.swring.count(img)) {
             for (int v = 0; v < V; v++) {
-                o << ind << ring(img, rs, 2 * v) << " = __byte_perm(__ldg(" << ptr << " + cl" << v << "), 0u, 0x4140);\n";
-                o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(__ldg(" << ptr << " + cl" << v << "), 0u, 0x4342);\n";
+                o << ind << ring(img, rs, 2 * v) << " = __byte_perm(KF_LDG(" << ptr << " + cl" << v << "), 0u, 0x4140);\n";
+                o << ind << ring(img, rs, 2 * v + 1) << " = __byte_perm(KF_LDG(" << ptr << " + cl" << v << "), 0u, 0x4342);\n";
             }
         } else {
             for (int v = 0; v < V; v++)
-                o << ind << ring(img, rs, v) << " = __ldg(" << ptr << " + cl" << v << ");\n";
+                o << ind << ring(img, rs, v) << " = KF_LDG(" << ptr << " + cl" << v << ");\n";
         }
     }
 
@@ -1558,8 +1558,8 @@ struct StreamGen {
     void bulk_row(const std::string &dst, const std::string &src, const std::string &guard, int s,
                   const std::string &ss, const std::string &ind)
     {
-        o << ind << "if (lane == 0 && " << guard << ") kf_bulk_row((char *)(" << dst << ") + toff, " << src << ", tb, "
-          << bar(s, ss) << ");\n";
+        o << ind << "if (lane == 0 && " << guard << ") { KF_RCHK(" << src << ", tb); kf_bulk_row((char *)(" << dst
+          << ") + toff, " << src << ", tb, " << bar(s, ss) << "); }\n";
     }
     void issue(int img, const std::string &ss, const std::string &it, const std::string &ind)
     {
@@ -1726,7 +1726,8 @@ struct StreamGen {
                 std::string val = f32 ? (pm ? sk[v] : ring(simg, ss, v))
                                       : si.swk.count(b.sink) ? ring(simg, ss, v)
                                                              : "kf_pack(" + val_memo[std::make_tuple(simg, ss, v)] + ")";
-                o << ind << "    if (x + " << v << " < a.fx1) (" << orow << ")[" << v << "] = " << val << ";\n";
+                o << ind << "    if (x + " << v << " < a.fx1 && KF_WOK(&(" << orow << ")[" << v << "], 4)) (" << orow << ")["
+                  << v << "] = " << val << ";\n";
             }
         } else if (f32) {
             for (int k = 0; k < NQ; k++) {
@@ -2131,6 +2132,10 @@ const OptDef kOpts[] = {
     // consumer tap -- the "pad once" fusion of Fig. 4b, which is WRONG at the
     // border.  Tests assert it fails parity.
     {"naive_border", 0, 0, 1, true},
+    // BOUNDS-CHECKING BUILD ONLY (libkfuse_bounds.so): the writable span of each
+    // launch loses its last output row, so the checker must report writes --
+    // its self-test.  The skipped row is then left unwritten.
+    {"bounds_shrink", 0, 0, 1, true},
 };
 #ifdef KF_EXPERIMENTAL
 constexpr bool kExperimental = true;
@@ -2142,11 +2147,17 @@ constexpr bool kTestHooks = true;
 #else
 constexpr bool kTestHooks = false;
 #endif
+#ifdef KF_BOUNDS
+constexpr bool kBounds = true;
+#else
+constexpr bool kBounds = false;
+#endif
 const OptDef *find_opt(const char *name)   // settable options of this build
 {
     for (const OptDef &d : kOpts)
         if (!std::strcmp(d.name, name)) {
             if (!std::strcmp(name, "naive_border")) return kTestHooks ? &d : nullptr;
+            if (!std::strcmp(name, "bounds_shrink")) return kBounds ? &d : nullptr;
             return (d.experimental && !kExperimental) ? nullptr : &d;
         }
     return nullptr;

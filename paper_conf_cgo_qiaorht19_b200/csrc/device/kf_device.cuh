@@ -29,6 +29,14 @@ struct KfArgs {
     int out_base;                  // global row held by row 0 of `out`
     int W, H;                      // image size (global)
     int r0, r1;                    // output rows computed by this launch
+#ifdef KF_BOUNDS
+    // bounds-checking build only (libkfuse_bounds.so): every
+    // global access is checked against these spans before it is made
+    unsigned long long span_lo[KF_MAX_IMG], span_hi[KF_MAX_IMG];   // readable: the external image buffers
+    unsigned long long out_lo, out_hi;                            // writable: this launch's output rows
+    int n_span;
+    unsigned *viol;                                               // [count, first addr lo, hi, is_write]
+#endif
     int indep;                     // 1: independent of the previous kernel on the stream (kf_run_batch
                                    // frames after the first): griddepcontrol.wait moves to the kernel's end
     // border frame: slow path, CTAs [0, frame_ctas)
@@ -171,34 +179,95 @@ __device__ __forceinline__ float kf_sel_gt(float a, float b, float c, float d) {
 __device__ __forceinline__ float kf_mac(float acc, float m, float v) { return fmaf(m, v, acc); }
 
 // ------------------------------------------------------ global image access
-__device__ __forceinline__ float kf_ldf(const void *p, int base, int W, int y, int x)
+__device__ __forceinline__ float kf_ldf_r(const void *p, int base, int W, int y, int x)
 {
     return __ldg((const float *)p + (size_t)(y - base) * W + x);
 }
-__device__ __forceinline__ I4 kf_ldi(const void *p, int base, int W, int y, int x)
+__device__ __forceinline__ I4 kf_ldi_r(const void *p, int base, int W, int y, int x)
 {
     return kf_unpack(__ldg((const unsigned *)p + (size_t)(y - base) * W + x));
 }
-__device__ __forceinline__ void kf_stf(void *p, int base, int W, int y, int x, float v)
+__device__ __forceinline__ void kf_stf_r(void *p, int base, int W, int y, int x, float v)
 {
     ((float *)p)[(size_t)(y - base) * W + x] = v;
 }
-__device__ __forceinline__ void kf_sti(void *p, int base, int W, int y, int x, I4 v)
+__device__ __forceinline__ void kf_sti_r(void *p, int base, int W, int y, int x, I4 v)
 {
     ((unsigned *)p)[(size_t)(y - base) * W + x] = kf_pack(v);
 }
 
 // 128-bit accesses of the streaming path (4 pixels per lane)
-__device__ __forceinline__ float4 kf_ld4f(const float *p) { return __ldg((const float4 *)p); }
-__device__ __forceinline__ uint4 kf_ld4u(const unsigned *p) { return __ldg((const uint4 *)p); }
-__device__ __forceinline__ void kf_st4f(float *p, float a, float b, float c, float d)
+__device__ __forceinline__ float4 kf_ld4f_r(const float *p) { return __ldg((const float4 *)p); }
+__device__ __forceinline__ uint4 kf_ld4u_r(const unsigned *p) { return __ldg((const uint4 *)p); }
+__device__ __forceinline__ void kf_st4f_r(float *p, float a, float b, float c, float d)
 {
     *(float4 *)p = make_float4(a, b, c, d);
 }
-__device__ __forceinline__ void kf_st4u(unsigned *p, unsigned a, unsigned b, unsigned c, unsigned d)
+__device__ __forceinline__ void kf_st4u_r(unsigned *p, unsigned a, unsigned b, unsigned c, unsigned d)
 {
     *(uint4 *)p = make_uint4(a, b, c, d);
 }
+
+// Access macros used by the generated code.  In the bounds-checking build
+// (KF_BOUNDS, libkfuse_bounds.so -- our stand-in for compute-sanitizer's
+// memcheck) every global read must fall inside one of the
+// launch's external image buffers and every write inside the launch's own
+// output rows; an access outside is skipped and counted (the first address is
+// kept) instead of faulting.  They expand where the launch arguments `a` are in
+// scope (every generated function).  Otherwise they are the plain accesses.
+#ifdef KF_BOUNDS
+__device__ __noinline__ bool kf_bchk(const KfArgs &a, const void *p, unsigned n, int wr)
+{
+    const unsigned long long x = (unsigned long long)p;
+    if (wr) {
+        if (x >= a.out_lo && x + n <= a.out_hi) return true;
+    } else {
+        for (int i = 0; i < a.n_span; i++)
+            if (x >= a.span_lo[i] && x + n <= a.span_hi[i]) return true;
+    }
+    if (atomicAdd(a.viol, 1u) == 0u) {
+        a.viol[1] = (unsigned)x;
+        a.viol[2] = (unsigned)(x >> 32);
+        a.viol[3] = (unsigned)wr;
+    }
+    return false;
+}
+__device__ __noinline__ int kf_bidx(const KfArgs &a, int i, int n)   // table index (LUT) in [0, n)
+{
+    if (i >= 0 && i < n) return i;
+    if (atomicAdd(a.viol, 1u) == 0u) { a.viol[1] = (unsigned)i; a.viol[2] = 0xffffffffu; a.viol[3] = 2u; }
+    return 0;
+}
+#define kf_ldf(p, base, W, y, x) \
+    (kf_bchk(a, (const float *)(p) + (size_t)((y) - (base)) * (W) + (x), 4, 0) ? kf_ldf_r(p, base, W, y, x) : 0.0f)
+#define kf_ldi(p, base, W, y, x) \
+    (kf_bchk(a, (const unsigned *)(p) + (size_t)((y) - (base)) * (W) + (x), 4, 0) ? kf_ldi_r(p, base, W, y, x) : kf_i4(0))
+#define kf_stf(p, base, W, y, x, v) \
+    do { if (kf_bchk(a, (float *)(p) + (size_t)((y) - (base)) * (W) + (x), 4, 1)) kf_stf_r(p, base, W, y, x, v); } while (0)
+#define kf_sti(p, base, W, y, x, v) \
+    do { if (kf_bchk(a, (unsigned *)(p) + (size_t)((y) - (base)) * (W) + (x), 4, 1)) kf_sti_r(p, base, W, y, x, v); } while (0)
+#define kf_ld4f(p) (kf_bchk(a, (p), 16, 0) ? kf_ld4f_r(p) : make_float4(0.f, 0.f, 0.f, 0.f))
+#define kf_ld4u(p) (kf_bchk(a, (p), 16, 0) ? kf_ld4u_r(p) : make_uint4(0u, 0u, 0u, 0u))
+#define kf_st4f(p, x0, x1, x2, x3) do { if (kf_bchk(a, (p), 16, 1)) kf_st4f_r((p), x0, x1, x2, x3); } while (0)
+#define kf_st4u(p, x0, x1, x2, x3) do { if (kf_bchk(a, (p), 16, 1)) kf_st4u_r((p), x0, x1, x2, x3); } while (0)
+#define KF_LDG(p) (kf_bchk(a, (p), (unsigned)sizeof(*(p)), 0) ? __ldg(p) : 0)
+#define KF_WOK(p, n) kf_bchk(a, (p), (n), 1)
+#define KF_IDX(i, n) kf_bidx(a, (int)(i), (n))
+#define KF_RCHK(p, n) ((void)kf_bchk(a, (p), (n), 0))
+#else
+#define kf_ldf kf_ldf_r
+#define kf_ldi kf_ldi_r
+#define kf_stf kf_stf_r
+#define kf_sti kf_sti_r
+#define kf_ld4f kf_ld4f_r
+#define kf_ld4u kf_ld4u_r
+#define kf_st4f kf_st4f_r
+#define kf_st4u kf_st4u_r
+#define KF_LDG(p) __ldg(p)
+#define KF_WOK(p, n) true
+#define KF_IDX(i, n) (i)
+#define KF_RCHK(p, n) ((void)0)
+#endif
 #define KF_FULL 0xffffffffu
 __device__ __forceinline__ float kf_shup(float v, int d) { return __shfl_up_sync(KF_FULL, v, d); }
 __device__ __forceinline__ float kf_shdn(float v, int d) { return __shfl_down_sync(KF_FULL, v, d); }
@@ -271,11 +340,16 @@ __device__ __forceinline__ F2 kf2_sel_gt(F2 a, F2 b, F2 c, F2 d)
 // Each streaming warp keeps DS input rows (512 B each) in flight in a shared
 // memory ring: 16 B per lane per row via cp.async (LDGSTS), one commit group
 // per row, consumed DS-1 groups later.
-__device__ __forceinline__ void kf_cp16(void *smem, const void *gmem)
+__device__ __forceinline__ void kf_cp16_r(void *smem, const void *gmem)
 {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
 }
+#ifdef KF_BOUNDS
+#define kf_cp16(d, g) do { if (kf_bchk(a, (g), 16, 0)) kf_cp16_r((d), (g)); } while (0)
+#else
+#define kf_cp16 kf_cp16_r
+#endif
 __device__ __forceinline__ void kf_cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N> __device__ __forceinline__ void kf_cp_wait()
 {

@@ -117,7 +117,11 @@ static std::string cache_dir()
 }
 
 static const char *kNvrtcOpts[] = {"--gpu-architecture=sm_100a", "-std=c++17", "-lineinfo", "-DKF_NVRTC=1",
-                                   "--extra-device-vectorization"};
+                                   "--extra-device-vectorization"
+#ifdef KF_BOUNDS
+                                   , "-DKF_BOUNDS=1"   // bounds-checking build: checked global accesses
+#endif
+};
 
 // NVRTC -> sm_100a cubin, cached on disk by hash(source, header, options).
 static std::string compile_cubin(const std::string &src, const std::string &name)
@@ -194,8 +198,10 @@ struct Runtime {
     // kf_run_host copy engines: H2D and D2H streams + per-band events
     cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
     cudaEvent_t ev_in[kHostBands] = {}, ev_out[kHostBands] = {}, ev_start = nullptr, ev_done = nullptr;
+    unsigned *viol = nullptr;   // bounds-checking build: violation record [count, addr lo, addr hi, kind]
     ~Runtime()
     {
+        if (viol) cudaFree(viol);
         for (void *q : stage_in) cudaFree(q);
         for (void *q : stage_out) cudaFree(q);
         for (int i = 0; i < kHostBands; i++) {
@@ -458,6 +464,25 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
             if (opt(p, "persist") && (long long)grid > slots) grid = (unsigned)slots;
         }
         if (grid == 0) continue;
+#ifdef KF_BOUNDS
+        {   // readable spans: each external image's buffer rows [base, rlast]; writable:
+            // this launch's output rows [r0, r1) (option bounds_shrink: minus the
+            // last row -- the checker's self-test, which must then report writes)
+            if (!p->rt->viol) {
+                KF_CUDA(cudaMalloc(&p->rt->viol, 4 * sizeof(unsigned)));
+                KF_CUDA(cudaMemset(p->rt->viol, 0, 4 * sizeof(unsigned)));
+            }
+            const unsigned long long rb = (unsigned long long)a.W * 4;
+            a.n_span = (int)b.ext.size();
+            for (size_t s2 = 0; s2 < b.ext.size(); s2++) {
+                a.span_lo[s2] = (unsigned long long)a.img[s2];
+                a.span_hi[s2] = a.span_lo[s2] + (unsigned long long)(a.rlast[s2] - a.base[s2] + 1) * rb;
+            }
+            a.out_lo = (unsigned long long)a.out + (unsigned long long)(a.r0 - a.out_base) * rb;
+            a.out_hi = (unsigned long long)a.out + (unsigned long long)(a.r1 - a.out_base - (opt(p, "bounds_shrink") ? 1 : 0)) * rb;
+            a.viol = p->rt->viol;
+        }
+#endif
         void *params[] = {&a};
         if (indep || opt(p, "pdl")) {
             // Programmatic dependent launch: this grid may be
@@ -646,6 +671,26 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
     KF_CUDA(cudaEventRecord(rt.ev_done, rt.s_d2h));
     KF_CUDA(cudaStreamWaitEvent(s, rt.ev_done, 0));
     KF_CUDA(cudaStreamSynchronize(s));
+}
+
+// Bounds-checking build: the pipeline's violation record (synchronises the
+// device).  Other builds have no checks: KF_ERR_ARG.
+void bounds_report(kf_pipeline *p, long long *count, unsigned long long *addr, int *kind)
+{
+#ifdef KF_BOUNDS
+    unsigned h[4] = {0, 0, 0, 0};
+    if (p->rt && p->rt->viol) {
+        KF_CUDA(cudaDeviceSynchronize());
+        KF_CUDA(cudaMemcpy(h, p->rt->viol, sizeof h, cudaMemcpyDeviceToHost));
+        KF_CUDA(cudaMemset(p->rt->viol, 0, sizeof h));
+    }
+    *count = h[0];
+    *addr = (unsigned long long)h[1] | ((unsigned long long)h[2] << 32);
+    *kind = (int)h[3];
+#else
+    (void)p; (void)count; (void)addr; (void)kind;
+    fail(KF_ERR_ARG, "bounds checks are compiled only into libkfuse_bounds.so");
+#endif
 }
 
 void release_plan(kf_plan *plan)

@@ -87,6 +87,7 @@ _SIGS = {
     "kf_prepare": (C.c_int, [_P, _P]),
     "kf_run": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_host": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
+    "kf_bounds_report": (C.c_int, [_P, C.POINTER(C.c_int64), C.POINTER(C.c_uint64), C.POINTER(C.c_int32)]),
     "kf_run_batch": (C.c_int, [_P, _P, C.c_int32, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_band": (C.c_int, [_P, _P, C.c_int32, C.c_int32, C.POINTER(_P), C.c_int32, C.c_int32,
                               C.POINTER(_P), _P]),
@@ -386,6 +387,13 @@ def peer_wait(counter, target, err, spin_limit=1 << 27, stream=None) -> None:
 def peer_enable(device: int, peer_device: int) -> None:
     """kf_peer_enable: kernels on `device` may access `peer_device`'s memory."""
     _check(lib.kf_peer_enable(int(device), int(peer_device)))
+
+
+def bounds_report(pipe: "Pipeline") -> tuple[int, int, int]:
+    """kf_bounds_report (bounds-checking build only): (violations, first address, kind)."""
+    n, ad, k = C.c_int64(), C.c_uint64(), C.c_int32()
+    _check(lib.kf_bounds_report(pipe.h, C.byref(n), C.byref(ad), C.byref(k)))
+    return n.value, ad.value, k.value
 
 
 def version() -> str:

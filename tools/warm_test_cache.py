@@ -94,19 +94,38 @@ def jobs():
     for o in ({"host_bands": 1}, {"host_bands": 3}, {"host_bands": 16}, {"host_bands": 32},
               {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}):
         out.append((P.harris(130, 1030), "b200", o, False))
+    # the bounds-checking build's launches (tests/test_bounds.py)
+    import importlib.util
+    bspec = importlib.util.spec_from_file_location("bounds_cases", os.path.join(ROOT, "tests", "bounds_cases.py"))
+    bc = importlib.util.module_from_spec(bspec)
+    bspec.loader.exec_module(bc)
+    for _, spec, kind, o in bc.cases():
+        out.append((spec, kind, o, "bounds"))
+    out.append((P.harris(300, 200), "b200", {"bounds_shrink": 1}, "bounds"))
+    for wl in ["harris", "deep10"]:
+        out.append((P.WORKLOADS[wl](300, 200), "b200", None, "bounds"))
+        out.append((P.WORKLOADS[wl](130, 1030), "b200", None, "bounds"))
     return out
 
 
+_MODS = {}
+
+
 def _mod(hooks):
+    """The product binding (hooks False), the test-hooks build (True) or the
+    bounds-checking build ("bounds")."""
     from paper_conf_cgo_qiaorht19_b200 import kfuse as K
     if not hooks:
         return K
-    import importlib.util
-    spec = importlib.util.spec_from_file_location("kfuse_testhooks", K.__file__)
-    m = importlib.util.module_from_spec(spec)
-    spec.loader.exec_module(m)
-    m.lib = m._open(os.path.join(os.path.dirname(K.__file__), "libkfuse_testhooks.so"))
-    return m
+    name = "libkfuse_bounds.so" if hooks == "bounds" else "libkfuse_testhooks.so"
+    if name not in _MODS:
+        import importlib.util
+        spec = importlib.util.spec_from_file_location("kfuse_" + name.split(".")[0], K.__file__)
+        m = importlib.util.module_from_spec(spec)
+        spec.loader.exec_module(m)
+        m.lib = m._open(os.path.join(os.path.dirname(K.__file__), name))
+        _MODS[name] = m
+    return _MODS[name]
 
 
 def compile_job(job):
