@@ -98,7 +98,7 @@ def _build_variant(lib_path: str, defs: list, force: bool, verbose: bool) -> str
             f.result()
     tmp = lib_path + f".{os.getpid()}.tmp"
     cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs + [
-        "-L/usr/local/cuda/lib64", "-lnvrtc", "-lcudart_static", "-ldl", "-lrt", "-lpthread",
+        "-L/usr/local/cuda/lib64", "-lnvrtc", "-lz", "-lcudart_static", "-ldl", "-lrt", "-lpthread",
         "-Xlinker", "-rpath=/usr/local/cuda/lib64"]
     if verbose:
         print(" ".join(cmd))

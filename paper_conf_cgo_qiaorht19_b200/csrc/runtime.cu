@@ -12,6 +12,7 @@
 #include <nvtx3/nvToolsExt.h>
 #include <sys/stat.h>
 #include <utime.h>
+#include <zlib.h>
 #include <unistd.h>
 
 #include <algorithm>
@@ -131,16 +132,25 @@ static std::string compile_cubin(const std::string &src, const std::string &name
     char hex[32];
     std::snprintf(hex, sizeof hex, "%016llx", (unsigned long long)fnv1a(key));
     const std::string dir = cache_dir();
-    const std::string path = dir + "/" + name + "_" + hex + ".cubin";
+    // zlib-compressed on disk ("KFZ1", uint64 size, deflate stream): the
+    // -lineinfo cubins of the unrolled kernels are 1-2.5 MB each and compress ~4x
+    const std::string path = dir + "/" + name + "_" + hex + ".cubin.z";
     {
         std::ifstream f(path, std::ios::binary);
         if (f) {
             std::stringstream ss;
             ss << f.rdbuf();
             std::string s = ss.str();
-            if (s.size() > 16) {
-                utime(path.c_str(), nullptr);   // mark as used (tools/warm_test_cache.py --prune keeps used cubins)
-                return s;
+            uint64_t n = 0;
+            if (s.size() > 12 && !s.compare(0, 4, "KFZ1")) {
+                std::memcpy(&n, s.data() + 4, 8);
+                std::string out(n, '\0');
+                uLongf got = (uLongf)n;
+                if (n > 16 && uncompress((Bytef *)&out[0], &got, (const Bytef *)s.data() + 12, (uLong)(s.size() - 12)) == Z_OK &&
+                    got == n) {
+                    utime(path.c_str(), nullptr);   // mark as used (tools/warm_test_cache.py --prune keeps used cubins)
+                    return out;
+                }
             }
         }
     }
@@ -168,8 +178,16 @@ static std::string compile_cubin(const std::string &src, const std::string &name
     std::string tmp = path + "." + std::to_string(getpid()) + "." +
                       std::to_string(std::hash<std::thread::id>()(std::this_thread::get_id())) + ".tmp";
     {
-        std::ofstream f(tmp, std::ios::binary);
-        if (f) f.write(cubin.data(), (std::streamsize)cubin.size());
+        uLongf zn = compressBound((uLong)cubin.size());
+        std::string z(12 + zn, '\0');
+        const uint64_t n = cubin.size();
+        std::memcpy(&z[0], "KFZ1", 4);
+        std::memcpy(&z[4], &n, 8);
+        if (compress2((Bytef *)&z[12], &zn, (const Bytef *)cubin.data(), (uLong)cubin.size(), 6) == Z_OK) {
+            z.resize(12 + zn);
+            std::ofstream f(tmp, std::ios::binary);
+            if (f) f.write(z.data(), (std::streamsize)z.size());
+        }
     }
     if (rename(tmp.c_str(), path.c_str()) != 0) unlink(tmp.c_str());
     return cubin;

@@ -180,9 +180,14 @@ def test_generated_kernels_compile_for_sm100a(seed, tmp_path, monkeypatch):
     p = K.Pipeline.from_spec(spec)
     plan = p.plan_fusion(rng.choice(["paper", "b200"]))
     plan.compile()
-    cubins = list(tmp_path.glob("*.cubin"))
+    cubins = list(tmp_path.glob("*.cubin.z"))   # zlib-compressed cache entries: "KFZ1", u64 size, deflate
     assert len(cubins) == len(plan.blocks)
-    blob = cubins[0].read_bytes()
+    import struct
+    import zlib
+    z = cubins[0].read_bytes()
+    assert z[:4] == b"KFZ1"
+    blob = zlib.decompress(z[12:])
+    assert len(blob) == struct.unpack("<Q", z[4:12])[0]
     assert blob[:4] == b"\x7fELF"
 
 

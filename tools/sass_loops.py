@@ -1,14 +1,23 @@
 """Instruction mix of the streaming loops of a cubin (diagnostics): every
 backward branch whose body holds warp shuffles, largest first.
 
-    python tools/sass_loops.py <file.cubin> [n]
+    python tools/sass_loops.py <file.cubin | kcache/*.cubin.z> [n]
 """
 import re
 import subprocess
 import sys
 from collections import Counter
 
-sass = subprocess.run(["cuobjdump", "-sass", sys.argv[1]], capture_output=True, text=True).stdout
+path = sys.argv[1]
+if path.endswith(".z"):   # a kcache entry: "KFZ1", u64 size, zlib stream
+    import tempfile
+    import zlib
+    with open(path, "rb") as f:
+        raw = zlib.decompress(f.read()[12:])
+    path = tempfile.mktemp(suffix=".cubin")
+    with open(path, "wb") as f:
+        f.write(raw)
+sass = subprocess.run(["cuobjdump", "-sass", path], capture_output=True, text=True).stdout
 ins = []
 for line in sass.splitlines():
     m = re.match(r"\s*/\*([0-9a-f]+)\*/\s*(.*?);", line)

@@ -26,7 +26,19 @@ def cubin_for(cfg: str, opts: dict) -> str:
             "spec, _ = P.config(%r)\n"
             "K.Pipeline.from_spec(spec, %r).plan_fusion('b200').compile()\n") % (ROOT, cfg, opts)
     subprocess.run([sys.executable, "-c", code], check=True, env=dict(os.environ, KFUSE_CACHE_DIR=d))
-    return os.path.join(d, [f for f in os.listdir(d) if f.endswith(".cubin")][0])
+    z = os.path.join(d, [f for f in os.listdir(d) if f.endswith(".cubin.z")][0])
+    return plain_cubin(z)
+
+
+def plain_cubin(path: str) -> str:
+    """A cache entry ("KFZ1", u64 size, zlib stream) decompressed next to it."""
+    import zlib
+    with open(path, "rb") as f:
+        z = f.read()
+    out = path[:-2] if path.endswith(".z") else path + ".cubin"
+    with open(out, "wb") as f:
+        f.write(zlib.decompress(z[12:]))
+    return out
 
 
 def summary(path: str) -> str:
