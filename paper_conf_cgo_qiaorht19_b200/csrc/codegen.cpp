@@ -1943,11 +1943,32 @@ struct StreamGen {
         loop_u0 = u0;
         if (si.rolled) {
             const int T = si.T;
-            o << "    #pragma unroll 1\n";
-            o << "    for (int u = " << u0 << "; u < nit; u += " << T << ") {\n";
-            if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
-            if (si.lpf) o << "        const int qnext = qb + " << T << " == " << si.DS << " ? 0 : qb + " << T << ";\n";
-            for (int j = 0; j < T; j++) iteration(j, -1, "u", "        ");
+            // warm_skip = 2: the iterations before every kernel is needed run in
+            // a loop of their own (guarded groups), so the
+            // steady-state loop carries no guards
+            int wend = u0;
+            if (opt(p, "warm_skip") == 2) {
+                for (int k : b.kernels) wend = std::max(wend, 2 * L - 2 * HY(p->n_inputs + k));
+                wend = u0 + (wend - u0 + T - 1) / T * T;
+            }
+            auto rolled_loop = [&](const std::string &hi, int guard_u0) {
+                loop_u0 = guard_u0;
+                o << "    #pragma unroll 1\n";
+                o << "    for (; u < " << hi << "; u += " << T << ") {\n";
+                if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
+                if (si.lpf) o << "        const int qnext = qb + " << T << " == " << si.DS << " ? 0 : qb + " << T << ";\n";
+                for (int j = 0; j < T; j++) iteration(j, -1, "u", "        ");
+                if (si.sring)
+                    o << "        qb += " << T << ";\n        if (qb == " << si.DS << ") { qb = 0;" << (tma ? " ph ^= 1u;" : "")
+                      << " }\n";
+                o << "    }\n";
+            };
+            o << "    int u = " << u0 << ";\n";
+            if (wend > u0) rolled_loop("min(nit, " + std::to_string(wend) + ")", u0);
+            rolled_loop("nit", wend);
+            o << "}\n\n";
+            runptr = false;
+            return;
         } else {
             o << "    for (int u = " << u0 << "; u < nit; u += " << P << ") {\n";
             if (si.sring) o << "        const int qprev = qb == 0 ? " << si.DS - 1 << " : qb - 1;\n";
@@ -2119,7 +2140,7 @@ const OptDef kOpts[] = {
     {"host_direct", 0, 0, 1, false},    // kf_run_host: kernels access pinned+mapped host buffers directly
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)
-    {"warm_skip", 1, 0, 1, false},      // loop warm-up rows skip kernels not yet needed (rolled bodies)
+    {"warm_skip", 2, 0, 2, false},      // rolled bodies: warm-up rows skip kernels not yet needed (1: guards in the loop, 2: own loop)
     {"pdl", 0, 0, 1, false},            // kf_run kernels launched as programmatic dependents (the CTA
                                         // launch overlaps the previous kernel's tail; measured mixed, off)
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
