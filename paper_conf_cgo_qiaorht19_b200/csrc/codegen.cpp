@@ -381,13 +381,22 @@ struct SwLin {
 };
 struct SwFail {};
 
+// SWAR table gathers of the interior path read a shared-memory copy of the
+// table (option lut_smem; filled once per CTA at kernel entry): a 32-bit LDS
+// address instead of 64-bit global address arithmetic per gather
+static bool lut_in_smem(const kf_pipeline *p, const Op &op)
+{
+    return !op.lut.empty() && op.lut.size() <= 1024 && opt(p, "lut_smem");
+}
+
 static long long floordiv(long long a, long long b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
 
 struct SwEmitter {
     std::ostringstream *o = nullptr;   // null: interval-only dry run (feasibility)
     int *tmp = nullptr;
     std::string ind;
-    std::string lut_sym;               // device table of the kernel being emitted (LUT ops)
+    std::string lut_sym;               // table of the kernel being emitted (LUT ops)
+    bool lut_shared = false;           // lut_sym is the CTA's shared-memory copy (plain indexing)
     std::string var() { return "w" + std::to_string((*tmp)++); }
     static std::string lit(long long v)   // v * 0x10001 as an unsigned literal (mod 2^32)
     {
@@ -550,8 +559,10 @@ struct SwEmitter {
             for (int c = 0; c < 4; c++) {
                 t[c] = var();
                 const std::string &w = c < 2 ? x.lo : x.hi;
-                *o << ind << "const unsigned " << t[c] << " = (unsigned)__ldg(" << lut_sym << " + KF_IDX("
-                   << (c % 2 ? "(" + w + " >> 16)" : "(" + w + " & 0xffffu)") << ", " << n << "));\n";
+                const std::string idx = "KF_IDX(" + (c % 2 ? "(" + w + " >> 16)" : "(" + w + " & 0xffffu)") + ", " +
+                                        std::to_string(n) + ")";
+                *o << ind << "const unsigned " << t[c] << " = (unsigned)"
+                   << (lut_shared ? lut_sym + "[" + idx + "]" : "__ldg(" + lut_sym + " + " + idx + ")") << ";\n";
             }
             r.lo = var();
             r.hi = var();
@@ -1234,6 +1245,10 @@ struct StreamGen {
         const int img = p->n_inputs + k;
         SwEmitter e = swe(ind);
         e.lut_sym = lut_sym(k);
+        if (lut_in_smem(p, op)) {
+            e.lut_sym = "kf_lutsh_" + std::to_string(block) + "_" + std::to_string(k);
+            e.lut_shared = true;
+        }
         std::vector<SwLin> res(V);
         if (op.kind == POINT) {
             for (int v = 0; v < V; v++) {
@@ -2140,6 +2155,7 @@ const OptDef kOpts[] = {
     {"host_direct", 0, 0, 1, false},    // kf_run_host: kernels access pinned+mapped host buffers directly
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)
+    {"lut_smem", 1, 0, 1, false},       // SWAR table gathers from a shared-memory copy of the table
     {"warm_skip", 2, 0, 2, false},      // rolled bodies: warm-up rows skip kernels not yet needed (1: guards in the loop, 2: own loop)
     {"pdl", 0, 0, 1, false},            // kf_run kernels launched as programmatic dependents (the CTA
                                         // launch overlaps the previous kernel's tail; measured mixed, off)
@@ -2380,6 +2396,8 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
             o << "__device__ const int kf_lut_" << block << "_" << k << "[" << p->ops[k].lut.size() << "] = {";
             for (size_t i = 0; i < p->ops[k].lut.size(); i++) o << (i ? "," : "") << p->ops[k].lut[i];
             o << "};\n";
+            if (lut_in_smem(p, p->ops[k]))
+                o << "__shared__ int kf_lutsh_" << block << "_" << k << "[" << p->ops[k].lut.size() << "];\n";
         }
     // one shared buffer per CTA: the frame path's staged tiles OR the interior
     // warp's input row rings (a CTA runs exactly one of the two paths)
@@ -2422,6 +2440,16 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     // completion of every earlier kernel on the stream.
     o << "    if (!a.indep) asm volatile(\"griddepcontrol.wait;\" ::: \"memory\");\n";
     o << "    asm volatile(\"griddepcontrol.launch_dependents;\");\n";
+    bool lut_fill = false;
+    for (int k : b.kernels)
+        if (lut_in_smem(p, p->ops[k])) {
+            const std::string n = std::to_string(p->ops[k].lut.size());
+            const std::string kb = std::to_string(block) + "_" + std::to_string(k);
+            o << "    for (int i = threadIdx.x; i < " << n << "; i += blockDim.x) kf_lutsh_" << kb << "[i] = kf_lut_" << kb
+              << "[i];\n";
+            lut_fill = true;
+        }
+    if (lut_fill) o << "    __syncthreads();\n";
     o << "    const int total = a.frame_ctas + (a.n_items + " << NW - 1 << ") / " << NW << ";\n";
     o << "    for (int cta = blockIdx.x; cta < total; cta += gridDim.x) {\n";
     o << "        if (cta < a.frame_ctas) " << kernel_name(block) << "_frame(a, cta);\n";
