@@ -1,4 +1,12 @@
-# r2e: calibration with the ROOFLINE (issue-rate) profile
+# r2e: evidence on the build with warm_skip=2 and lut_smem -- GPU suite, smoke, bench, reference arm, ncu launch list, ncu --set full of C3 and C4
 mkdir -p gpurun_out
-timeout 2400 python tools/calibrate.py --out gpurun_out/calibration_r2e.json > gpurun_out/calibrate_r2e.log 2>&1; echo "calibrate rc=$?"
-tail -8 gpurun_out/calibrate_r2e.log | cut -c1-900
+KF_PARITY_LOG=gpurun_out/parity_r2e.jsonl timeout 1500 python -m pytest tests -q -m gpu > gpurun_out/tests_r2e.log 2>&1; echo "tests rc=$?"; tail -2 gpurun_out/tests_r2e.log
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_r2e.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/smoke_r2e.log
+timeout 900 python bench.py --steps 200 --warmup 5 > gpurun_out/bench_r2e.json 2> gpurun_out/bench_r2e.err; echo "bench rc=$?"; head -c 300 gpurun_out/bench_r2e.json
+timeout 600 python bench.py --impl reference --steps 5 --warmup 3 > gpurun_out/bench_ref_r2e.json 2>&1; echo "ref rc=$?"
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv --log-file gpurun_out/r02_launches_c3_e.csv python bench.py --steps 20 --warmup 3 --no-extra --no-cpu > gpurun_out/ncu_launch_bench_e.log 2>&1; echo "ncu launches rc=$?"
+for cfg in C3 C4; do
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:kf_b -s 2 -c 1 -f -o gpurun_out/r02_${cfg}_b200_full_e \
+     python tools/prof_run.py --config $cfg --plan b200 > gpurun_out/ncu_${cfg}_e.log 2>&1; echo "ncu $cfg rc=$?"
+done
+python tools/ncu_extract.py C3=gpurun_out/r02_C3_b200_full_e.ncu-rep C4=gpurun_out/r02_C4_b200_full_e.ncu-rep > gpurun_out/r02_ncu_c3_c4_e.json; echo "extract rc=$?"
