@@ -949,6 +949,8 @@ struct StreamGen {
     std::map<std::tuple<int, int, int>, std::string> val_memo;
     std::map<std::tuple<std::string, int, int>, std::string> shfl_memo;   // (var, lane offset, edge key)
     std::map<std::tuple<int, int, int>, SwReg> sw_memo;                     // SWAR values (image, slot, column)
+    std::map<std::pair<int, int>, std::string> dl_memo;                      // delay-line rows read (image, age)
+    std::string cur_it = "0";                                                // iteration index of the body being emitted
     std::map<int, int> xe;   // pair mode: deferred power-of-two exponent of each image's stored values
     int xe_of(int img) const { auto it = xe.find(img); return pm && it != xe.end() ? it->second : 0; }
     void set_xe(int img, int e)
@@ -1186,6 +1188,19 @@ struct StreamGen {
         auto key = std::make_tuple(img, s, v);
         auto it = sw_memo.find(key);
         if (it != sw_memo.end()) return it->second;
+        if (si.delay.count(img) && s >= si.depth.at(img)) {   // row older than the register ring: delay line
+            auto dk = std::make_pair(img, s);
+            if (!dl_memo.count(dk)) {
+                const std::string t = var();
+                o << ind << "const uint4 " << t << " = dl" << img << "[((" << cur_it << " - " << s << ") & "
+                  << si.delay.at(img) - 1 << ") * 32];\n";
+                dl_memo[dk] = t;
+            }
+            const char *c[4] = {"x", "y", "z", "w"};
+            SwReg r = swe(ind).unpack(dl_memo[dk] + "." + c[v]);
+            sw_memo[key] = r;
+            return r;
+        }
         if (si.swring.count(img)) {   // SWAR ring: already unpacked (bias 0, [0, 255])
             SwReg r;
             r.lo = ring(img, s, 2 * v);
@@ -1318,6 +1333,11 @@ struct StreamGen {
                 o << ind << ring(img, ws, v) << " = " << e.pack(r) << ";\n";
             }
             sw_memo[std::make_tuple(img, ws, v)] = r;
+        }
+        if (si.delay.count(img)) {   // the packed row into the kernel's delay line, slot (iteration mod S)
+            o << ind << "dl" << img << "[(" << cur_it << " & " << si.delay.at(img) - 1 << ") * 32] = make_uint4(";
+            for (int v = 0; v < V; v++) o << (v ? ", " : "") << ring(img, ws, v);
+            o << ");\n";
         }
     }
 
@@ -1613,6 +1633,8 @@ struct StreamGen {
                 o << ind << "const " << (f32 ? "float4 " : "uint4 ") << q[k] << " = *(" << slot_ptr(s, ss) << " + " << k << ");\n";
         }
         unpack_row(img, rs, q, ind);
+        if (si.delay.count(img))   // the packed row into the image's delay line, slot (iteration mod S)
+            o << ind << "dl" << img << "[(" << cur_it << " & " << si.delay.at(img) - 1 << ") * 32] = " << q[0] << ";\n";
     }
 
     // One iteration (slot j).  u >= 0: peeled edge iteration with index u.
@@ -1622,8 +1644,10 @@ struct StreamGen {
         val_memo.clear();
         shfl_memo.clear();
         sw_memo.clear();
+        dl_memo.clear();
         swsh_memo.clear();
         o << ind.substr(2) << "{   // iteration " << uexpr << " + " << j << "\n";
+        cur_it = u >= 0 ? std::to_string(u) : "(" + uexpr + " + " + std::to_string(j) + ")";
         if (si.sring) {
             const int DS = si.DS;
             std::string s_iss, s_get;
@@ -1694,7 +1718,7 @@ struct StreamGen {
             if (g != group) {
                 if (group >= 0) {
                     o << ind << "}\n";
-                    val_memo.clear(); shfl_memo.clear(); sw_memo.clear(); swsh_memo.clear();
+                    val_memo.clear(); shfl_memo.clear(); sw_memo.clear(); swsh_memo.clear(); dl_memo.clear();
                 }
                 if (g >= 0) o << ind << "if (" << uexpr << " + " << j << " >= " << first << ") {\n";
                 group = g;
@@ -1703,7 +1727,7 @@ struct StreamGen {
         }
         if (group >= 0) {
             o << ind << "}\n";
-            val_memo.clear(); shfl_memo.clear(); sw_memo.clear(); swsh_memo.clear();
+            val_memo.clear(); shfl_memo.clear(); sw_memo.clear(); swsh_memo.clear(); dl_memo.clear();
         }
         const int simg = p->n_inputs + b.sink;
         const int ss = sl(simg, 0, j);
@@ -1869,6 +1893,9 @@ struct StreamGen {
                 o << "    " << (f32 ? "float4" : "uint4") << " *sr" << s << " = (" << (f32 ? "float4" : "uint4")
                   << " *)(" << kernel_name(block) << "_smem + " << s * si.DS * 512 * NQ << " + wslot) + lane * " << NQ << ";\n";
             }
+            for (auto &kv : si.delay)   // shared-memory delay lines (stream_info)
+                o << "    uint4 *dl" << kv.first << " = (uint4 *)(" << kernel_name(block) << "_smem + "
+                  << si.delay_off.at(kv.first) << " + wslot) + lane;\n";
             if (tma) {
                 // one mbarrier per (image, ring slot) after the rings.  The warp's
                 // row segment is lanes 0..31's columns [x0w, x0w + 32V) clipped to
@@ -2155,6 +2182,7 @@ const OptDef kOpts[] = {
     {"host_direct", 0, 0, 1, false},    // kf_run_host: kernels access pinned+mapped host buffers directly
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)
+    {"delay_smem", 1, 0, 1, false},     // rolled u8x4 bodies: far point-read rows from shared-memory delay lines
     {"lut_smem", 1, 0, 1, false},       // SWAR table gathers from a shared-memory copy of the table
     {"warm_skip", 2, 0, 2, false},      // rolled bodies: warm-up rows skip kernels not yet needed (1: guards in the loop, 2: own loop)
     {"pdl", 0, 0, 1, false},            // kf_run kernels launched as programmatic dependents (the CTA
@@ -2289,6 +2317,70 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         si.tma = si.sring && opt(p, "tma");
     }
     if (!si.sring) si.P = std::max(maxdepth, maxdepth_ext + si.D);
+    // code size: scalar operations of one iteration (one body copy)
+    long long ops = 0;
+    for (int k : b.kernels) {
+        const Op &op = p->ops[k];
+        const int ch = p->dtype == KF_F32 ? 1 : si.swk.count(k) ? 2 : 4;   // SWAR: two channels per op
+        if (op.kind == LOCAL) {
+            int nnz = 0;
+            for (double m : op.mask) nnz += m != 0.0;
+            const Separable &sp = si.sep.at(k);
+            int taps = sp.ok ? (int)(std::count_if(sp.col.begin(), sp.col.end(), [](double c) { return c != 0.0; }) +
+                                     std::count_if(sp.row.begin(), sp.row.end(), [](double c) { return c != 0.0; }))
+                             : nnz;
+            ops += (long long)(taps + 2 * op.rx() + prog_size(op)) * kV_ * ch;
+        } else {
+            ops += (long long)prog_size(op) * kV_ * ch;
+        }
+    }
+    si.iter_ops = ops;
+    // unrolled: ~P copies per variant (4 variants + 2 peeled prologues); too
+    // much straight-line code for NVRTC/ptxas and the instruction cache ->
+    // one rolled body copy
+    const long long budget = opt(p, "code_budget");
+    si.rolled = ops * si.P * 6 > budget;
+    // rows per rolled trip (option rtrip): 2 halves the ring-shift moves; the
+    // shared-memory ring then holds a multiple of T rows (slot qb + j < DS)
+    si.T = si.rolled && si.sring ? (int)opt(p, "rtrip") : 1;
+    if (si.T > 1) {
+        while (si.DS % si.T) si.DS += si.P;
+        if (si.DS % si.T) si.DS = si.DS * si.T;
+        si.ring_bytes = (int)b.ext.size() * si.DS * 128 * kV_;
+    }
+    // Shared-memory delay lines (option delay_smem): in a rolled
+    // body every ring row is a register shifted by a move each iteration.  An
+    // image whose deepest rows are read only by SWAR point kernels (a value
+    // carried to the sink row: deep10's input for k7/k9, k0 for k8) keeps only
+    // the rows its local consumers' windows read in registers; the older rows
+    // come from a per-warp shared-memory line of S rows (packed, 16 B per lane,
+    // row of iteration t in slot t mod S).  Fewer moves and registers, which
+    // lets the next ring stay unpacked under the register cap.
+    if (p->dtype == KF_U8X4 && si.rolled && si.T == 1 && si.sring && !si.tma && opt(p, "delay_smem")) {
+        int off = si.ring_bytes;
+        for (auto &kv : si.depth) {
+            const int img = kv.first, full = kv.second;
+            if (img == p->n_inputs + b.sink) continue;
+            const bool ext = std::binary_search(b.ext.begin(), b.ext.end(), img);
+            if (!ext && !si.swk.count(img - p->n_inputs)) continue;   // SWAR producer (packed row at hand)
+            int wdepth = 1;
+            bool ok = true;
+            for (int k : b.kernels) {
+                const Op &op = p->ops[k];
+                if (std::find(op.inputs.begin(), op.inputs.end(), img) == op.inputs.end()) continue;
+                if (!si.swk.count(k)) ok = false;   // far rows are read through the SWAR path only
+                if (op.kind == LOCAL) wdepth = std::max(wdepth, si.hy[img] - si.hy[p->n_inputs + k] + op.ry() + 1);
+            }
+            if (!ok || full - wdepth < 2) continue;
+            int S = 1;
+            while (S < full) S *= 2;
+            si.delay[img] = S;
+            si.delay_off[img] = off;
+            off += S * 32 * 16;
+            kv.second = wdepth;
+        }
+        si.ring_bytes = off;
+    }
     // register estimate: live ring values (depth per image, D prefetched rows)
     int live = 0;
     for (auto &kv : si.depth) {
@@ -2308,6 +2400,7 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
             const int img = kv.first;
             if (img == p->n_inputs + b.sink || kv.second < 3) continue;
             const bool ext = std::binary_search(b.ext.begin(), b.ext.end(), img);
+            if (!ext && si.delay.count(img)) continue;   // its delay line stores the packed row
             if (!ext && !si.swk.count(img - p->n_inputs)) continue;   // producer must be SWAR (or a load)
             bool vert = false;
             for (int k : b.kernels)
@@ -2324,24 +2417,6 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         }
     }
     si.live_regs = live;
-    // code size: scalar operations of one iteration (one body copy)
-    long long ops = 0;
-    for (int k : b.kernels) {
-        const Op &op = p->ops[k];
-        const int ch = p->dtype == KF_F32 ? 1 : si.swk.count(k) ? 2 : 4;   // SWAR: two channels per op
-        if (op.kind == LOCAL) {
-            int nnz = 0;
-            for (double m : op.mask) nnz += m != 0.0;
-            const Separable &sp = si.sep.at(k);
-            int taps = sp.ok ? (int)(std::count_if(sp.col.begin(), sp.col.end(), [](double c) { return c != 0.0; }) +
-                                     std::count_if(sp.row.begin(), sp.row.end(), [](double c) { return c != 0.0; }))
-                             : nnz;
-            ops += (long long)(taps + 2 * op.rx() + prog_size(op)) * kV_ * ch;
-        } else {
-            ops += (long long)prog_size(op) * kV_ * ch;
-        }
-    }
-    si.iter_ops = ops;
     // image edges inside the streaming path: not for REPEAT
     // (wrap reads the opposite side), horizontal only when every exterior tap of
     // the edge lane maps into its own 4 pixels
@@ -2353,19 +2428,6 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
         hfit &= op.rx() <= (op.mode == KF_MIRROR101 ? kV_ - 1 : kV_);
     }
     si.edge_v = !rep && p->H >= 4 * si.L + 2 * si.P + 8;
-    // unrolled: ~P copies per variant (4 variants + 2 peeled prologues); too
-    // much straight-line code for NVRTC/ptxas and the instruction cache ->
-    // one rolled body copy
-    const long long budget = opt(p, "code_budget");
-    si.rolled = ops * si.P * 6 > budget;
-    // rows per rolled trip (option rtrip): 2 halves the ring-shift moves; the
-    // shared-memory ring then holds a multiple of T rows (slot qb + j < DS)
-    si.T = si.rolled && si.sring ? (int)opt(p, "rtrip") : 1;
-    if (si.T > 1) {
-        while (si.DS % si.T) si.DS += si.P;
-        if (si.DS % si.T) si.DS = si.DS * si.T;
-        si.ring_bytes = (int)b.ext.size() * si.DS * 128 * kV_;
-    }
     // rolled bodies keep the edge strips too (peeled remapped prologue, then
     // the rolled loop), unless option rolled_edge_v=0 leaves those rows to the
     // frame: for deep10 the frame's index-exchange tiles cost 12 % of the kernel

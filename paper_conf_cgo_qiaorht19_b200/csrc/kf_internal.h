@@ -172,6 +172,8 @@ struct StreamInfo {
     std::map<int, Separable> sep; // local kernel -> factorisation
     std::set<int> swk;            // u8x4 kernels in SWAR form (two channels per 32-bit op)
     std::set<int> swring;         // u8x4 images whose ring holds the unpacked SWAR (lo, hi) pair
+    std::map<int, int> delay;     // u8x4 image -> rows S of its shared-memory delay line (option delay_smem)
+    std::map<int, int> delay_off; // image -> byte offset of that line within the warp's shared memory
 };
 
 std::string kernel_name(const BlockInfo &b, int block);

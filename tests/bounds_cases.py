@@ -21,7 +21,8 @@ def cases():
             for size in [(45, 37), (5, 5), (33, 17)]:
                 out.append((f"{wl}-{mode}-{size[0]}x{size[1]}", P.WORKLOADS[wl](*size, mode=mode), "b200", None))
     for o in ({"tma": 1}, {"cta_warps": 4}, {"code_budget": 1000}, {"smem_rows": 6}, {"sring": 0},
-              {"peel_warmup": 0}, {"rtrip": 2, "code_budget": 1000}, {"warm_skip": 0}, {"warm_skip": 1}):
+              {"peel_warmup": 0}, {"rtrip": 2, "code_budget": 1000}, {"warm_skip": 0}, {"warm_skip": 1},
+              {"delay_smem": 0}, {"code_budget": 1000, "warm_skip": 1}):
         tag = ",".join(f"{k}={v}" for k, v in o.items())
         for wl in ["harris", "deep10", "unsharp"]:
             out.append((f"{wl}-200x150-{tag}", P.WORKLOADS[wl](200, 150), "b200", o))
