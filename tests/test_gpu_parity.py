@@ -122,6 +122,18 @@ def test_workloads_all_border_modes_fused(wl, mode):
         assert plan.num_launches == 1
 
 
+@pytest.mark.parametrize("mode", P.MODES)
+@pytest.mark.parametrize("size", [(128, 96), (516, 70)])
+@pytest.mark.parametrize("wl", ["deep10", "swar_stress"])
+def test_rolled_streaming_all_border_modes(wl, mode, size):
+    """The rolled u8x4 streaming path with every vector-path feature on -- the
+    cp.async ring, the separate warm-up loop, the shared-memory LUT and delay
+    lines -- at widths that take it (W % 4 == 0), under every border mode, edge
+    strips and edge chunks included: bit-exact against the oracle."""
+    spec = P.WORKLOADS[wl](*size, mode=mode) if wl != "swar_stress" else P.swar_stress(*size, mode=mode)
+    parity(spec, "b200")
+
+
 def test_fig4_fused_on_gpu():
     """Fig. 4c through the fused GPU kernel: 763 at (0,0), 992 at (2,2)."""
     spec = P.fig4("clamp")
