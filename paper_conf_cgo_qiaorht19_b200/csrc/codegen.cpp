@@ -2191,6 +2191,7 @@ const OptDef kOpts[] = {
     {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
     {"persist_waves", 1, 1, 1 << 20, true},
     {"nlong", 0, 0, 1 << 20, true},     // tail split (rejected)
+    {"cluster", 1, 1, 8, true},         // thread-block clusters of this many CTAs (CTA-dispatch experiment)
     // NEGATIVE CONTROL ONLY: settable in libkfuse_testhooks.so (KF_TEST_HOOKS),
     // never in the product library, where it is always 0.  The frame path then
     // evaluates in-block producers on the padded plane instead of remapping each

@@ -502,7 +502,9 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         }
 #endif
         void *params[] = {&a};
-        if (indep || opt(p, "pdl")) {
+        const bool pdl = indep || opt(p, "pdl");
+        const int cluster = (int)opt(p, "cluster");   // experimental: thread-block clusters of this many CTAs
+        if (pdl || cluster > 1) {
             // Programmatic dependent launch: this grid may be
             // scheduled once every CTA of the previous kernel on the stream has
             // triggered (this library's kernels trigger after their own wait).
@@ -511,10 +513,20 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
             // launch overlaps the previous tail.  An independent frame of
             // kf_run_batch runs concurrently with the previous frame's tail and
             // waits for it at its end.
-            CUlaunchAttribute attr[1];
+            CUlaunchAttribute attr[2];
             std::memset(attr, 0, sizeof attr);
-            attr[0].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
-            attr[0].value.programmaticStreamSerializationAllowed = 1;
+            unsigned na = 0;
+            if (pdl) {
+                attr[na].id = CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION;
+                attr[na++].value.programmaticStreamSerializationAllowed = 1;
+            }
+            if (cluster > 1) {   // grid rounded up to whole clusters; surplus CTAs find no work
+                grid = (grid + cluster - 1) / cluster * cluster;
+                attr[na].id = CU_LAUNCH_ATTRIBUTE_CLUSTER_DIMENSION;
+                attr[na].value.clusterDim.x = (unsigned)cluster;
+                attr[na].value.clusterDim.y = 1;
+                attr[na++].value.clusterDim.z = 1;
+            }
             CUlaunchConfig cfg;
             std::memset(&cfg, 0, sizeof cfg);
             cfg.gridDimX = grid; cfg.gridDimY = 1; cfg.gridDimZ = 1;
@@ -522,7 +534,7 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
             cfg.sharedMemBytes = 0;
             cfg.hStream = st;
             cfg.attrs = attr;
-            cfg.numAttrs = 1;
+            cfg.numAttrs = na;
             cu_check(d.launchKernelEx(&cfg, cb.fn, params, nullptr), "cuLaunchKernelEx");
         } else {
             cu_check(d.launchKernel(cb.fn, grid, 1, 1, kThreads * cb.si.nw, 1, 1, 0, st, params, nullptr),
