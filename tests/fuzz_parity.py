@@ -10,8 +10,9 @@ front in parallel.
 
     python tests/fuzz_parity.py [n_dags] [seed0] [oracle|bands]   -> one JSON line, exit 1 on any mismatch
 
-Mode `bands` checks the decompositions instead: kf_run_host and random row
-bands (kf_run_band) against the whole-image kf_run, bit for bit.
+Mode `bands` checks the decompositions instead: kf_run_host, random row
+bands (kf_run_band) and three kf_run_batch frames against the whole-image
+kf_run, bit for bit.
 """
 import json
 import os
@@ -31,7 +32,12 @@ from oracle import oracle as O  # noqa: E402
 from paper_conf_cgo_qiaorht19_b200 import kfuse as K  # noqa: E402
 
 OPTIONS = [{}, {}, {}, {"tma": 1}, {"rtrip": 2}, {"cta_warps": 4}, {"code_budget": 1000}, {"peel_warmup": 0},
-           {"lds_pf": 0}, {"qptr": 0}, {"sring": 0}, {"swring": 0}, {"smem_rows": 6}, {"heavy_first": 0}]
+           {"lds_pf": 0}, {"qptr": 0}, {"sring": 0}, {"swring": 0}, {"smem_rows": 6}, {"heavy_first": 0},
+           # rolled bodies (small code budget): separate warm-up loop, shared-memory LUT and delay lines, and their
+           # alternatives; programmatic dependent launch
+           {"code_budget": 1000}, {"code_budget": 1000}, {"code_budget": 1000, "warm_skip": 1},
+           {"code_budget": 1000, "warm_skip": 0}, {"code_budget": 1000, "delay_smem": 0},
+           {"code_budget": 1000, "lut_smem": 0}, {"pdl": 1}]
 
 
 def case(i, seed0):
@@ -101,6 +107,12 @@ def bands_mode(cases):
                 plan.run_band(r0, r1, b_in, a0, a1, b_out)
                 torch.cuda.synchronize()
                 ok &= all(np.array_equal(o.cpu().numpy(), f[r0:r1]) for o, f in zip(b_out, full))
+        if ok:   # three independent frames through kf_run_batch (overlapping launches when single-block)
+            fin = [[torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in ins] for _ in range(3)]
+            fout = [[torch.empty(shape, dtype=dt, device="cuda") for _ in spec["outputs"]] for _ in range(3)]
+            plan.run_batch(fin, fout)
+            torch.cuda.synchronize()
+            ok &= all(np.array_equal(o.cpu().numpy(), f) for fo in fout for o, f in zip(fo, full))
         if not ok:
             bad.append({"seed": seed, "kind": kind, "opts": opts, "size": [W, H], "dtype": spec["dtype"]})
     return bad
