@@ -383,10 +383,12 @@ struct SwFail {};
 
 // SWAR table gathers of the interior path read a shared-memory copy of the
 // table (option lut_smem; filled once per CTA at kernel entry): a 32-bit LDS
-// address instead of 64-bit global address arithmetic per gather
-static bool lut_in_smem(const kf_pipeline *p, const Op &op)
+// address instead of 64-bit global address arithmetic per gather.  Decided
+// per block by stream_info (si.lut_smem), which keeps the CTA's static shared
+// memory -- rings or frame tiles plus the tables -- within 48 KB.
+static bool lut_in_smem(const StreamInfo &si, const Op &op)
 {
-    return !op.lut.empty() && op.lut.size() <= 1024 && opt(p, "lut_smem");
+    return si.lut_smem && !op.lut.empty() && op.lut.size() <= 1024;
 }
 
 static long long floordiv(long long a, long long b) { return a >= 0 ? a / b : -((-a + b - 1) / b); }
@@ -1260,7 +1262,7 @@ struct StreamGen {
         const int img = p->n_inputs + k;
         SwEmitter e = swe(ind);
         e.lut_sym = lut_sym(k);
-        if (lut_in_smem(p, op)) {
+        if (lut_in_smem(si, op)) {
             e.lut_sym = "kf_lutsh_" + std::to_string(block) + "_" + std::to_string(k);
             e.lut_shared = true;
         }
@@ -2438,7 +2440,21 @@ StreamInfo stream_info(const kf_pipeline *p, const BlockInfo &b)
     si.ok = b.Rx <= 2 * kV_ * 4 && live_packed <= 160 && b.ext.size() <= KF_MAX_IMG_HOST;
     si.warp_smem = (si.ring_bytes + (si.tma ? 8 * (int)b.ext.size() * si.DS : 0) + 15) / 16 * 16;
     // warps per CTA, capped so the CTA's static shared buffer stays within 48 KB
-    si.nw = std::max(1, std::min((int)opt(p, "cta_warps"), 49152 / std::max(si.warp_smem, 1)));
+    // shared-memory copies of small tables (option lut_smem) share the CTA's
+    // 48 KB of static shared memory with the rings (or the frame tiles)
+    int lut_bytes = 0;
+    if (opt(p, "lut_smem"))
+        for (int k : b.kernels)
+            if (!p->ops[k].lut.empty() && p->ops[k].lut.size() <= 1024) lut_bytes += 4 * (int)p->ops[k].lut.size();
+    si.nw = std::max(1, std::min((int)opt(p, "cta_warps"), (49152 - lut_bytes) / std::max(si.warp_smem, 1)));
+    int frame_bytes = 0;
+    for (int k : b.staged) {
+        int n = 0;
+        for (int s2 = 0; s2 < 2; s2++)
+            n = std::max(n, (kFrameTiles[s2][0] + 2 * b.hx.at(k)) * (kFrameTiles[s2][1] + 2 * b.hy.at(k)));
+        frame_bytes += n * 4;
+    }
+    si.lut_smem = lut_bytes > 0 && std::max(frame_bytes, si.nw * si.warp_smem) + lut_bytes <= 49152;
     if (opt(p, "naive_border")) si.ok = false;   // negative control: everything through the (naive) frame
     return si;
 }
@@ -2459,7 +2475,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
             o << "__device__ const int kf_lut_" << block << "_" << k << "[" << p->ops[k].lut.size() << "] = {";
             for (size_t i = 0; i < p->ops[k].lut.size(); i++) o << (i ? "," : "") << p->ops[k].lut[i];
             o << "};\n";
-            if (lut_in_smem(p, p->ops[k]))
+            if (lut_in_smem(si, p->ops[k]))
                 o << "__shared__ int kf_lutsh_" << block << "_" << k << "[" << p->ops[k].lut.size() << "];\n";
         }
     // one shared buffer per CTA: the frame path's staged tiles OR the interior
@@ -2505,7 +2521,7 @@ std::string generate_block(const kf_pipeline *p, const BlockInfo &b, int block)
     o << "    asm volatile(\"griddepcontrol.launch_dependents;\");\n";
     bool lut_fill = false;
     for (int k : b.kernels)
-        if (lut_in_smem(p, p->ops[k])) {
+        if (lut_in_smem(si, p->ops[k])) {
             const std::string n = std::to_string(p->ops[k].lut.size());
             const std::string kb = std::to_string(block) + "_" + std::to_string(k);
             o << "    for (int i = threadIdx.x; i < " << n << "; i += blockDim.x) kf_lutsh_" << kb << "[i] = kf_lut_" << kb

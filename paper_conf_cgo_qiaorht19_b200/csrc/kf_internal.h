@@ -174,6 +174,7 @@ struct StreamInfo {
     std::set<int> swring;         // u8x4 images whose ring holds the unpacked SWAR (lo, hi) pair
     std::map<int, int> delay;     // u8x4 image -> rows S of its shared-memory delay line (option delay_smem)
     std::map<int, int> delay_off; // image -> byte offset of that line within the warp's shared memory
+    bool lut_smem = false;        // small tables gathered from shared-memory copies (option lut_smem)
 };
 
 std::string kernel_name(const BlockInfo &b, int block);
