@@ -27,6 +27,22 @@ _spec.loader.exec_module(BC)
 CASES = BC.cases()
 
 
+@pytest.fixture(scope="module", autouse=True)
+def _precompile_kernels():
+    """Compiles this module's kernels (bounds-checking build) up front in parallel
+    threads: instant when build() warmed the in-tree cubin cache."""
+    from concurrent.futures import ThreadPoolExecutor
+    root = os.path.dirname(_HERE)
+    spec = importlib.util.spec_from_file_location("warm_test_cache", os.path.join(root, "tools", "warm_test_cache.py"))
+    w = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(w)
+    jobs = [j for j in w.jobs() if j[3] == "bounds"]
+    jobs += [(spec, kind, opts, False) for _, spec, kind, opts in CASES]   # product twins
+    with ThreadPoolExecutor(max(1, min(32, os.cpu_count() or 1))) as ex:
+        list(ex.map(w.compile_job, jobs))
+    yield
+
+
 @pytest.fixture(scope="module")
 def B():
     """A second binding instance bound to the bounds-checking build."""

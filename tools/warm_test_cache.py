@@ -107,6 +107,7 @@ def jobs():
     bspec.loader.exec_module(bc)
     for _, spec, kind, o in bc.cases():
         out.append((spec, kind, o, "bounds"))
+        out.append((spec, kind, o, False))   # the product twin each bounds-checked result is compared with
     out.append((P.harris(300, 200), "b200", {"bounds_shrink": 1}, "bounds"))
     for wl in ["harris", "deep10"]:
         out.append((P.WORKLOADS[wl](300, 200), "b200", None, "bounds"))
