@@ -193,11 +193,14 @@ kf_status kf_mark_output(kf_pipeline *p, int32_t image_id);
  * plans prepared afterwards; run-time options (nstrips, host_taper) at the next
  * kf_run.  Names: swar swring swring_cap prefetch sring smem_rows lds_pf
  * const_w pro_rp qptr heavy_first code_budget rolled_edge_v minctas nstrips
- * host_taper host_bands host_direct tma rtrip cta_warps peel_warmup pdl.  Unknown names or out-of-range values: KF_ERR_ARG.
- * (The measured-and-rejected v8 / persist / persist_waves / nlong and the
- * rounding-changing diagnostics pairs / defer exist only in a KF_EXPERIMENTAL
- * build, and the naive_border negative control only in the KF_TEST_HOOKS build
- * libkfuse_testhooks.so, never in libkfuse.so.) */
+ * host_taper host_bands host_direct tma rtrip cta_warps peel_warmup pdl
+ * warm_skip lut_smem delay_smem.  Unknown names or out-of-range values:
+ * KF_ERR_ARG.  (The measured-and-rejected v8 / persist / persist_waves / nlong
+ * / cluster and the rounding-changing diagnostics pairs / defer exist only in
+ * a KF_EXPERIMENTAL build, the naive_border negative control only in the
+ * KF_TEST_HOOKS build libkfuse_testhooks.so, and the bounds_shrink self-test
+ * only in the bounds-checking build libkfuse_bounds.so -- never in
+ * libkfuse.so.) */
 kf_status kf_set_option(kf_pipeline *p, const char *name, int64_t value);
 kf_status kf_get_option(const kf_pipeline *p, const char *name, int64_t *value);
 
