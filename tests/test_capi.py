@@ -290,6 +290,52 @@ def test_swar_form_chosen_by_interval_analysis():
     assert "kf_unpack" not in src and "kf_lut(" not in src   # all ten deep10 kernels in SWAR form
 
 
+def _di(src: str) -> str:
+    """The interior variant of a generated block (the hot loop's function)."""
+    body = src.split("_fast_di(")[1]
+    return body[:body.index("\n}\n")]
+
+
+def test_rolled_u8x4_codegen_choices():
+    """What the code generator decides for deep10 (C4, a rolled u8x4 body), read
+    from the generated source: the warm-up rows run in a
+    loop of their own and the steady-state loop carries no guards (warm_skip=2);
+    warm_skip=1 puts warp-uniform guards into the one loop; the LUT is gathered
+    from a shared-memory copy; the input and k0 keep their far rows in
+    shared-memory delay lines, which frees the registers for k4's unpacked ring;
+    f32 pipelines and option delay_smem=0 get none."""
+    c4, _ = P.config("C4")
+    src = K.Pipeline.from_spec(c4).plan_fusion("b200").source(0)
+    di = _di(src)
+    assert "for (; u < min(nit, 12); u += 1)" in di and "for (; u < nit; u += 1)" in di
+    steady = di[di.index("for (; u < nit; u += 1)"):]
+    assert "if (u + 0 >= " not in steady
+    assert "__shared__ int kf_lutsh_0_6[256];" in src and "kf_lutsh_0_6[KF_IDX(" in di
+    assert "uint4 *dl0 = " in di and "uint4 *dl1 = " in di                  # input and k0 delay lines
+    assert "- 6) & 7) * 32]" in di and "- 4) & 7) * 32]" in di              # ages 6 and 4 read from them
+    assert "live~152" in src.splitlines()[0]
+    guarded = _di(K.Pipeline.from_spec(c4, {"warm_skip": 1}).plan_fusion("b200").source(0))
+    assert "for (; u < min(nit," not in guarded and "if (u + 0 >= 12) {" in guarded
+    no_dl = K.Pipeline.from_spec(c4, {"delay_smem": 0}).plan_fusion("b200").source(0)
+    assert "uint4 *dl" not in no_dl and "live~164" in no_dl.splitlines()[0]
+    no_lut = K.Pipeline.from_spec(c4, {"lut_smem": 0}).plan_fusion("b200").source(0)
+    assert "kf_lutsh_" not in no_lut and "__ldg(kf_lut_0_6 + KF_IDX(" in no_lut
+    f32 = K.Pipeline.from_spec(P.enhance(2048, 2048)).plan_fusion("b200").source(0)
+    assert "rolled" in f32.splitlines()[0] and "uint4 *dl" not in f32
+
+
+def test_shared_luts_fit_static_shared_memory():
+    """Shared-memory table copies are dropped when rings x warps per CTA plus the
+    tables would exceed 48 KB of static shared memory (found by the fuzz: a LUT
+    under cta_warps=4)."""
+    c4, _ = P.config("C4")
+    one = K.Pipeline.from_spec(c4).plan_fusion("b200").source(0)
+    assert "kf_lutsh_" in one
+    many = K.Pipeline.from_spec(c4, {"cta_warps": 8}).plan_fusion("b200").source(0)
+    m = re.search(r"_smem\[(\d+)\]", many)
+    assert m and int(m.group(1)) + (1024 if "kf_lutsh_" in many else 0) <= 49152
+
+
 def test_schedule_options_api():
     """kf_set_option / kf_get_option: known options with defaults and ranges; unknown
     names, out-of-range values and the test-only / experimental options are
