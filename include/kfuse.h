@@ -193,7 +193,7 @@ kf_status kf_mark_output(kf_pipeline *p, int32_t image_id);
  * plans prepared afterwards; run-time options (nstrips, host_taper) at the next
  * kf_run.  Names: swar swring swring_cap prefetch sring smem_rows lds_pf
  * const_w pro_rp qptr heavy_first code_budget rolled_edge_v minctas nstrips
- * host_taper host_bands host_direct tma rtrip cta_warps peel_warmup pdl
+ * host_taper host_bands host_async_bands host_direct tma rtrip cta_warps peel_warmup pdl
  * warm_skip lut_smem delay_smem.  Unknown names or out-of-range values:
  * KF_ERR_ARG.  (The measured-and-rejected v8 / persist / persist_waves / nlong
  * / cluster and the rounding-changing diagnostics pairs / defer exist only in
@@ -310,6 +310,19 @@ kf_status kf_bounds_report(kf_pipeline *p, int64_t *violations, uint64_t *first_
  * owned by the pipeline.  Work already queued on `stream` precedes the copies. */
 kf_status kf_run_host(kf_pipeline *p, const kf_plan *plan, const void *const *h_inputs, int32_t n_in,
                       void *const *h_outputs, int32_t n_out, void *stream);
+
+/* kf_run_host without the final synchronisation, for a stream of host images:
+ * returns once the work is queued; the outputs are in host memory when
+ * `stream`'s work completes (its later work is ordered after the downloads).
+ * Consecutive calls alternate between two device staging sets, so call k+1's
+ * uploads overlap call k's downloads (the copy engines run both directions at
+ * once).  Unlike kf_run_host, the uploads are NOT ordered after work already
+ * queued on `stream`: the host inputs must be ready at the call and must not
+ * be written by pending work, and inputs and outputs must stay untouched until
+ * the stream's work completes.  Host buffers must be pinned.  Results equal
+ * kf_run's bit for bit. */
+kf_status kf_run_host_async(kf_pipeline *p, const kf_plan *plan, const void *const *h_inputs, int32_t n_in,
+                            void *const *h_outputs, int32_t n_out, void *stream);
 
 /* Row-band execution for the multi-GPU layer: computes output rows
  * [row0, row1) of every marked output into d_out_band[j] (rows row0.. at

@@ -382,6 +382,15 @@ kf_status kf_run_host(kf_pipeline *p, const kf_plan *plan, const void *const *h_
     });
 }
 
+kf_status kf_run_host_async(kf_pipeline *p, const kf_plan *plan, const void *const *h_inputs, int32_t n_in,
+                            void *const *h_outputs, int32_t n_out, void *stream)
+{
+    return guard([&] {
+        if (!p || !plan || plan->pipe != p) fail(KF_ERR_ARG, "plan does not belong to pipeline");
+        run_host(p, const_cast<kf_plan *>(plan), h_inputs, n_in, h_outputs, n_out, stream, true);
+    });
+}
+
 kf_status kf_run_band(kf_pipeline *p, const kf_plan *plan, int32_t row0, int32_t row1,
                       const void *const *d_in_band, int32_t in_row0, int32_t in_row1, void *const *d_out_band,
                       void *stream)

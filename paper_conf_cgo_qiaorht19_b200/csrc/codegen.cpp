@@ -2181,6 +2181,7 @@ const OptDef kOpts[] = {
     {"nstrips", 0, 0, 1 << 20, false},  // force the strip count (0 = cost model)
     {"host_taper", 1, 0, 1, false},     // kf_run_host thin first/last bands
     {"host_bands", 8, 1, 32, false},    // kf_run_host row bands (pipeline depth)
+    {"host_async_bands", 2, 1, 32, false},   // kf_run_host_async row bands
     {"host_direct", 0, 0, 1, false},    // kf_run_host: kernels access pinned+mapped host buffers directly
     {"tma", 0, 0, 1, false},            // interior rows fed by TMA bulk copies + mbarriers (§5.5)
     {"cta_warps", 1, 1, 8, false},      // interior warps (items) per CTA (frame tiles use all of them)

@@ -192,7 +192,7 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
 void run_batch(kf_pipeline *p, kf_plan *plan, int n_frames, const void *const *din, int n_in,
                void *const *dout, int n_out, void *stream);
 void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
-              void *stream);
+              void *stream, bool async = false);
 void bounds_report(kf_pipeline *p, long long *count, unsigned long long *addr, int *kind);
 void release_plan(kf_plan *plan);
 void release_runtime(kf_pipeline *p);

@@ -210,18 +210,23 @@ constexpr int kHostBands = 32;  // kf_run_host: most row bands (option host_band
 
 struct Runtime {
     std::map<uint64_t, std::shared_ptr<CompiledBlock>> modules;   // by source hash
-    std::vector<void *> stage_in, stage_out;                      // kf_run_host staging
+    std::vector<void *> stage_in[2], stage_out[2];                // kf_run_host staging (2 sets: async calls alternate)
     size_t stage_bytes = 0;
     int device = -1;
     // kf_run_host copy engines: H2D and D2H streams + per-band events
     cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
     cudaEvent_t ev_in[kHostBands] = {}, ev_out[kHostBands] = {}, ev_start = nullptr, ev_done = nullptr;
+    cudaEvent_t ev_kern[2] = {};   // kf_run_host_async: the kernels that read staging set s are done
+    size_t async_calls = 0;
     unsigned *viol = nullptr;   // bounds-checking build: violation record [count, addr lo, addr hi, kind]
     ~Runtime()
     {
         if (viol) cudaFree(viol);
-        for (void *q : stage_in) cudaFree(q);
-        for (void *q : stage_out) cudaFree(q);
+        for (int k = 0; k < 2; k++) {
+            for (void *q : stage_in[k]) cudaFree(q);
+            for (void *q : stage_out[k]) cudaFree(q);
+            if (ev_kern[k]) cudaEventDestroy(ev_kern[k]);
+        }
         for (int i = 0; i < kHostBands; i++) {
             if (ev_in[i]) cudaEventDestroy(ev_in[i]);
             if (ev_out[i]) cudaEventDestroy(ev_out[i]);
@@ -592,7 +597,7 @@ void run_batch(kf_pipeline *p, kf_plan *plan, int n_frames, const void *const *d
 // Band k waits only for the input rows it reads, [row0 - R, row1 + R).
 // REPEAT plans (no band mode) and tiny images run as one band.
 void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, void *const *hout, int n_out,
-              void *stream)
+              void *stream, bool async)
 {
     if (n_in != p->n_inputs || n_out != (int)p->outputs.size()) fail(KF_ERR_ARG, "wrong number of buffers");
     prepare(p, plan);
@@ -620,23 +625,36 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
         for (int j = 0; j < n_out && ok; j++) ok = mapped(hout[j], &dq[j]);
         if (ok) {
             run(p, plan, di.data(), n_in, dq.data(), n_out, stream, 0, p->H, 0, p->H);
-            KF_CUDA(cudaStreamSynchronize((cudaStream_t)stream));
+            if (!async) KF_CUDA(cudaStreamSynchronize((cudaStream_t)stream));
             return;
         }
     }
     Runtime &rt = *p->rt;
     const size_t row_bytes = (size_t)p->W * 4, bytes = row_bytes * p->H;
-    if (rt.stage_bytes != bytes || rt.stage_in.size() != (size_t)n_in || rt.stage_out.size() != (size_t)n_out) {
-        for (void *q : rt.stage_in) cudaFree(q);
-        for (void *q : rt.stage_out) cudaFree(q);
-        rt.stage_in.assign(n_in, nullptr);
-        rt.stage_out.assign(n_out, nullptr);
-        for (auto &q : rt.stage_in)
-            if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
-        for (auto &q : rt.stage_out)
-            if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
+    // Staging set: the synchronous call uses set 0; asynchronous calls alternate
+    // between two sets, so call k+1 uploads into one set while call k's kernels
+    // and download still use the other.
+    const int set = async ? (int)(rt.async_calls++ % 2) : 0;
+    if (rt.stage_bytes != bytes) {
+        for (int k = 0; k < 2; k++) {
+            for (void *q : rt.stage_in[k]) cudaFree(q);
+            for (void *q : rt.stage_out[k]) cudaFree(q);
+            rt.stage_in[k].clear();
+            rt.stage_out[k].clear();
+        }
         rt.stage_bytes = bytes;
     }
+    if (rt.stage_in[set].size() != (size_t)n_in || rt.stage_out[set].size() != (size_t)n_out) {
+        for (void *q : rt.stage_in[set]) cudaFree(q);
+        for (void *q : rt.stage_out[set]) cudaFree(q);
+        rt.stage_in[set].assign(n_in, nullptr);
+        rt.stage_out[set].assign(n_out, nullptr);
+        for (auto &q : rt.stage_in[set])
+            if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
+        for (auto &q : rt.stage_out[set])
+            if (cudaMalloc(&q, bytes) != cudaSuccess) fail(KF_ERR_OOM, "staging allocation failed");
+    }
+    std::vector<void *> &stage_in = rt.stage_in[set], &stage_out = rt.stage_out[set];
     if (!rt.s_h2d) {
         KF_CUDA(cudaStreamCreateWithFlags(&rt.s_h2d, cudaStreamNonBlocking));
         KF_CUDA(cudaStreamCreateWithFlags(&rt.s_d2h, cudaStreamNonBlocking));
@@ -646,18 +664,30 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
         }
         KF_CUDA(cudaEventCreateWithFlags(&rt.ev_start, cudaEventDisableTiming));
         KF_CUDA(cudaEventCreateWithFlags(&rt.ev_done, cudaEventDisableTiming));
+        for (int k = 0; k < 2; k++) KF_CUDA(cudaEventCreateWithFlags(&rt.ev_kern[k], cudaEventDisableTiming));
     }
     cudaStream_t s = (cudaStream_t)stream;
     bool repeat = false;
     for (const auto &op : p->ops) repeat |= op.kind == LOCAL && op.mode == KF_REPEAT;
     const int R = plan->halo_rows;
-    const int want = std::min(kHostBands, (int)opt(p, "host_bands"));
+    // bands per call: 8 for a synchronous call (its first upload and last
+    // download are exposed; thin end bands shorten them), 2 for an asynchronous
+    // one (consecutive calls hide each other's ends; fewer, larger copies)
+    const int want = std::min(kHostBands, (int)opt(p, async ? "host_async_bands" : "host_bands"));
     int nb = repeat ? 1 : std::max(1, std::min(want, p->H / std::max(64, 4 * R)));
-    std::vector<const void *> din(rt.stage_in.begin(), rt.stage_in.end());
-    // the copy streams start after everything already queued on the caller's stream
-    KF_CUDA(cudaEventRecord(rt.ev_start, s));
-    KF_CUDA(cudaStreamWaitEvent(rt.s_h2d, rt.ev_start, 0));
-    KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_start, 0));
+    std::vector<const void *> din(stage_in.begin(), stage_in.end());
+    if (!async) {
+        // the copy streams start after everything already queued on the caller's stream
+        KF_CUDA(cudaEventRecord(rt.ev_start, s));
+        KF_CUDA(cudaStreamWaitEvent(rt.s_h2d, rt.ev_start, 0));
+        KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_start, 0));
+    } else {
+        // asynchronous: the upload into this set waits only for the kernels that
+        // read it two calls ago (the caller guarantees the host inputs are ready);
+        // its download buffers were released when the caller's stream waited for
+        // that call's downloads
+        KF_CUDA(cudaStreamWaitEvent(rt.s_h2d, rt.ev_kern[set], 0));
+    }
     int copied = 0;   // input rows [0, copied) are queued on the H2D stream
     // Band boundaries.  Only the first band's upload and the last band's
     // download are exposed (everything else overlaps), so with 8 bands the
@@ -678,7 +708,7 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
         const int need = k == nb - 1 ? p->H : std::min(p->H, r1 + R);
         if (need > copied) {
             for (int i = 0; i < n_in; i++)
-                KF_CUDA(cudaMemcpyAsync((char *)rt.stage_in[i] + copied * row_bytes,
+                KF_CUDA(cudaMemcpyAsync((char *)stage_in[i] + copied * row_bytes,
                                         (const char *)hin[i] + copied * row_bytes, (need - copied) * row_bytes,
                                         cudaMemcpyHostToDevice, rt.s_h2d));
             copied = need;
@@ -687,7 +717,7 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
         KF_CUDA(cudaStreamWaitEvent(s, rt.ev_in[k], 0));
         // the band writes rows [r0, r1) of the whole staging image (out_full): a
         // pointer offset to row r0 would not be 16-B aligned when W % 4 != 0
-        std::vector<void *> dout(rt.stage_out.begin(), rt.stage_out.end());
+        std::vector<void *> dout(stage_out.begin(), stage_out.end());
         if (nb == 1)
             run(p, plan, din.data(), n_in, dout.data(), n_out, stream, 0, p->H, 0, p->H);
         else
@@ -695,12 +725,13 @@ void run_host(kf_pipeline *p, kf_plan *plan, const void *const *hin, int n_in, v
         KF_CUDA(cudaEventRecord(rt.ev_out[k], s));
         KF_CUDA(cudaStreamWaitEvent(rt.s_d2h, rt.ev_out[k], 0));
         for (int j = 0; j < n_out; j++)
-            KF_CUDA(cudaMemcpyAsync((char *)hout[j] + r0 * row_bytes, (const char *)rt.stage_out[j] + r0 * row_bytes,
+            KF_CUDA(cudaMemcpyAsync((char *)hout[j] + r0 * row_bytes, (const char *)stage_out[j] + r0 * row_bytes,
                                     (r1 - r0) * row_bytes, cudaMemcpyDeviceToHost, rt.s_d2h));
     }
+    KF_CUDA(cudaEventRecord(rt.ev_kern[set], s));
     KF_CUDA(cudaEventRecord(rt.ev_done, rt.s_d2h));
     KF_CUDA(cudaStreamWaitEvent(s, rt.ev_done, 0));
-    KF_CUDA(cudaStreamSynchronize(s));
+    if (!async) KF_CUDA(cudaStreamSynchronize(s));
 }
 
 // Bounds-checking build: the pipeline's violation record (synchronises the

@@ -88,6 +88,7 @@ _SIGS = {
     "kf_run": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_host": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_bounds_report": (C.c_int, [_P, C.POINTER(C.c_int64), C.POINTER(C.c_uint64), C.POINTER(C.c_int32)]),
+    "kf_run_host_async": (C.c_int, [_P, _P, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_batch": (C.c_int, [_P, _P, C.c_int32, C.POINTER(_P), C.c_int32, C.POINTER(_P), C.c_int32, _P]),
     "kf_run_band": (C.c_int, [_P, _P, C.c_int32, C.c_int32, C.POINTER(_P), C.c_int32, C.c_int32,
                               C.POINTER(_P), _P]),
@@ -345,6 +346,11 @@ class Plan:
         """End-to-end: host numpy/pinned-tensor buffers in and out (kf_run_host)."""
         _check(lib.kf_run_host(self.pipe.h, self.h, _ptrs([_dptr(t) for t in inputs]), len(inputs),
                                _ptrs([_dptr(t) for t in outputs]), len(outputs), _P(_stream(stream))))
+
+    def run_host_async(self, inputs, outputs, stream=None) -> None:
+        """kf_run_host_async: pinned host buffers; no final synchronisation."""
+        _check(lib.kf_run_host_async(self.pipe.h, self.h, _ptrs([_dptr(t) for t in inputs]), len(inputs),
+                                     _ptrs([_dptr(t) for t in outputs]), len(outputs), _P(_stream(stream))))
 
     def run_band(self, row0, row1, in_band, in_row0, in_row1, out_band, stream=None) -> None:
         _check(lib.kf_run_band(self.pipe.h, self.h, int(row0), int(row1),

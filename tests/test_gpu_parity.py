@@ -343,6 +343,50 @@ def test_run_batch_rejects_shared_outputs():
     torch.cuda.synchronize()
 
 
+@pytest.mark.parametrize("wl,kind,size", [("harris", "b200", (300, 200)), ("deep10", "b200", (260, 150)),
+                                          ("harris", "unfused", (130, 1030)), ("two_input", "b200", (512, 300)),
+                                          ("harris", "b200", (130, 97))])
+def test_run_host_async_stream_of_images(wl, kind, size):
+    """kf_run_host_async over a stream of images (consecutive calls alternate two
+    staging sets; uploads of call k+1 overlap downloads of call k) == kf_run per
+    image, bit for bit; mixed with a synchronous kf_run_host in the middle."""
+    spec = P.WORKLOADS[wl](*size)
+    plan = make_plan(spec, kind)
+    n = 5
+    frames = [_inputs(spec, 60 + f) for f in range(n)]
+    refs = [run_gpu(spec, plan, ins) for ins in frames]
+    hin = [[torch.from_numpy(np.ascontiguousarray(a)).pin_memory() for a in ins] for ins in frames]
+    hout = [[torch.zeros(r.shape, dtype=torch.float32 if spec["dtype"] == "f32" else torch.uint8).pin_memory()
+             for r in ref] for ref in refs]
+    st = torch.cuda.Stream()
+    for f in range(n):
+        if f == 2:
+            plan.run_host(hin[f], hout[f], st)
+        else:
+            plan.run_host_async(hin[f], hout[f], st)
+    st.synchronize()
+    for f in range(n):
+        for g, r in zip(hout[f], refs[f]):
+            np.testing.assert_array_equal(g.numpy(), r, err_msg=f"image {f}")
+
+
+@pytest.mark.parametrize("nb", [1, 3, 8])
+def test_run_host_async_band_counts(nb):
+    """Any kf_run_host_async band count (option host_async_bands) gives kf_run's bits."""
+    spec = P.harris(130, 1030)
+    plan = make_plan(spec, "b200", {"host_async_bands": nb})
+    frames = [_inputs(spec, 80 + f) for f in range(3)]
+    refs = [run_gpu(spec, plan, ins)[0] for ins in frames]
+    hin = [torch.from_numpy(np.ascontiguousarray(f[0])).pin_memory() for f in frames]
+    hout = [torch.zeros(r.shape, dtype=torch.float32).pin_memory() for r in refs]
+    st = torch.cuda.Stream()
+    for f in range(3):
+        plan.run_host_async([hin[f]], [hout[f]], st)
+    st.synchronize()
+    for f in range(3):
+        np.testing.assert_array_equal(hout[f].numpy(), refs[f])
+
+
 def test_run_host_repeat_and_pinned():
     """REPEAT plans (one band) and pinned host buffers on a non-default stream."""
     spec = P.harris(256, 300, "repeat")

@@ -96,6 +96,10 @@ def jobs():
     for o in ({"host_bands": 1}, {"host_bands": 3}, {"host_bands": 16}, {"host_bands": 32},
               {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}):
         out.append((P.harris(130, 1030), "b200", o, False))
+    out.append((P.deep10(260, 150), "b200", None, False))
+    out.append((P.two_input(512, 300), "b200", None, False))
+    out.append((P.harris(130, 97), "b200", None, False))
+    out.append((P.harris(130, 1030), "unfused", None, False))
     for mode in P.MODES:
         for size in [(128, 96), (516, 70)]:
             out.append((P.deep10(*size, mode=mode), "b200", None, False))
