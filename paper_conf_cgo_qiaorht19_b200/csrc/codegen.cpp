@@ -2188,8 +2188,9 @@ const OptDef kOpts[] = {
     {"delay_smem", 1, 0, 1, false},     // rolled u8x4 bodies: far point-read rows from shared-memory delay lines
     {"lut_smem", 1, 0, 1, false},       // SWAR table gathers from a shared-memory copy of the table
     {"warm_skip", 2, 0, 2, false},      // rolled bodies: warm-up rows skip kernels not yet needed (1: guards in the loop, 2: own loop)
-    {"pdl", 0, 0, 1, false},            // kf_run kernels launched as programmatic dependents (the CTA
-                                        // launch overlaps the previous kernel's tail; measured mixed, off)
+    {"pdl", 2, 0, 2, false},            // kf_run kernels launched as programmatic dependents (the CTA
+                                        // launch overlaps the previous kernel's tail): 0 off, 1 all,
+                                        // 2 unrolled blocks (rolled C4 measured slower)
     {"v8", 0, 0, 1, true},              // 8 pixels per lane (rejected, §5.4)
     {"persist", 0, 0, 1, true},         // persistent CTAs (rejected)
     {"persist_waves", 1, 1, 1 << 20, true},

@@ -507,7 +507,11 @@ void run(kf_pipeline *p, kf_plan *plan, const void *const *din, int n_in, void *
         }
 #endif
         void *params[] = {&a};
-        const bool pdl = indep || opt(p, "pdl");
+        // option pdl: 0 off, 1 every launch, 2 (default) every launch of an
+        // unrolled block -- measured faster on every memory-bound config, but
+        // slower on the compute-bound rolled C4 kernel
+        const long long pdl_opt = opt(p, "pdl");
+        const bool pdl = indep || pdl_opt == 1 || (pdl_opt == 2 && !cb.si.rolled);
         const int cluster = (int)opt(p, "cluster");   // experimental: thread-block clusters of this many CTAs
         if (pdl || cluster > 1) {
             // Programmatic dependent launch: this grid may be

@@ -681,7 +681,7 @@ SAME_BITS = [{"qptr": 0}, {"lds_pf": 0}, {"const_w": 0}, {"heavy_first": 0}, {"p
              {"peel_warmup": 0}, {"peel_warmup": 0, "lds_pf": 0}, {"pdl": 1},
              {"warm_skip": 0}, {"warm_skip": 0, "code_budget": 1000}, {"warm_skip": 1},
              {"warm_skip": 1, "code_budget": 1000}, {"pdl": 1, "code_budget": 1000}, {"lut_smem": 0},
-             {"delay_smem": 0}, {"delay_smem": 1, "code_budget": 1000}]
+             {"delay_smem": 0}, {"delay_smem": 1, "code_budget": 1000}, {"pdl": 0}]
 EXPERIMENTAL = [{"v8": 1}, {"persist": 1}, {"nlong": 3}, {"persist": 1, "persist_waves": 2}, {"cluster": 4}]
 # experimental options that change the f32 rounding (scalar instead of packed pairs,
 # scales applied per stage): within the parity tolerance of the oracle, not bit-identical

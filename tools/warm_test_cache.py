@@ -58,7 +58,7 @@ def jobs():
             {"peel_warmup": 0}, {"peel_warmup": 0, "lds_pf": 0}, {"pdl": 1},
             {"warm_skip": 0}, {"warm_skip": 0, "code_budget": 1000}, {"warm_skip": 1},
             {"warm_skip": 1, "code_budget": 1000}, {"pdl": 1, "code_budget": 1000}, {"lut_smem": 0},
-            {"delay_smem": 0}, {"delay_smem": 1, "code_budget": 1000}]
+            {"delay_smem": 0}, {"delay_smem": 1, "code_budget": 1000}, {"pdl": 0}]
     exp = [{"v8": 1}, {"persist": 1}, {"nlong": 3}]
     for wl in ["harris", "unsharp", "shitomasi"]:
         for o in ({"pairs": 0}, {"defer": 0}):
