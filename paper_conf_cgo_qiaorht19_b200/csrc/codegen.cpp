@@ -1240,6 +1240,12 @@ struct StreamGen {
             else m = edge_map(op.mode, -(q - V) - 1);
             if (m < 0) {
                 slo = shi = SwEmitter::lit(csub + row[0].B);
+                // the border constant may lie outside the row's interval (a
+                // producer whose values are provably >= 128, a constant 0):
+                // the bias analysis downstream must see it, or a sum that goes
+                // negative only at the image edge wraps a 16-bit lane
+                t.vlo = std::min(t.vlo, csub);
+                t.vhi = std::max(t.vhi, csub);
             } else {
                 const SwReg &sr = q < 0 ? row[m] : row[V - 1 - m];
                 slo = sr.lo;
