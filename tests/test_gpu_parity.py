@@ -134,6 +134,26 @@ def test_rolled_streaming_all_border_modes(wl, mode, size):
     parity(spec, "b200")
 
 
+@pytest.mark.parametrize("width", [130, 128, 516])
+@pytest.mark.parametrize("opts", [{}, {"code_budget": 1000}])
+def test_swar_constant_border_below_producer_range(width, opts):
+    """Regression (fuzz seed 1020420): a fused point -> local pair where the point
+    kernel's values are provably >= 128 and the local kernel's CONSTANT border is
+    0.  The edge lane substitutes the constant, which lies outside the producer's
+    interval; the SWAR bias must cover it or a sum that is negative only at the
+    image edge wraps a 16-bit lane (x = 0 came out 255 instead of 0)."""
+    p = P.Pipeline("constant_edge", width, 17, "u8x4")
+    i = p.input()
+    a = p.point("p3", [i], [P.L(0), P.C(3), P.MUL, P.SHR(2), P.SAT])
+    b = p.point("p4", [a, i], [P.L(0), P.L(1), P.ADD, P.C(128), P.ADD, P.SAT])
+    p.output(p.local("l5", b, [[16, -8, 8]], "constant", constant=0.0,
+                     post=[P.L(0), P.C(16), P.ADD, P.SHR(5), P.C(0), P.ADD, P.SAT]))
+    spec = p.spec()
+    ins = _inputs(spec, 7)
+    got = run_gpu(spec, make_plan(spec, "b200", opts), ins)[0]
+    check(spec, got, O.run(spec, ins)[spec["outputs"][0]], f"constant_edge {width} {opts}")
+
+
 def test_fig4_fused_on_gpu():
     """Fig. 4c through the fused GPU kernel: 763 at (0,0), 992 at (2,2)."""
     spec = P.fig4("clamp")

@@ -96,6 +96,15 @@ def jobs():
     for o in ({"host_bands": 1}, {"host_bands": 3}, {"host_bands": 16}, {"host_bands": 32},
               {"host_bands": 12, "host_taper": 0}, {"host_direct": 1}):
         out.append((P.harris(130, 1030), "b200", o, False))
+    for width in (130, 128, 516):   # test_swar_constant_border_below_producer_range
+        p = P.Pipeline("constant_edge", width, 17, "u8x4")
+        i = p.input()
+        a = p.point("p3", [i], [P.L(0), P.C(3), P.MUL, P.SHR(2), P.SAT])
+        b = p.point("p4", [a, i], [P.L(0), P.L(1), P.ADD, P.C(128), P.ADD, P.SAT])
+        p.output(p.local("l5", b, [[16, -8, 8]], "constant", constant=0.0,
+                         post=[P.L(0), P.C(16), P.ADD, P.SHR(5), P.C(0), P.ADD, P.SAT]))
+        for o in (None, {"code_budget": 1000}):
+            out.append((p.spec(), "b200", o, False))
     out.append((P.deep10(260, 150), "b200", None, False))
     out.append((P.two_input(512, 300), "b200", None, False))
     out.append((P.harris(130, 97), "b200", None, False))
