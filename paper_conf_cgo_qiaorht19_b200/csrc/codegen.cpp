@@ -949,7 +949,10 @@ struct StreamGen {
     std::map<int, int> slot;   // external image -> slot
     // per-iteration memo: (image, ring slot, column) -> unpacked value variable
     std::map<std::tuple<int, int, int>, std::string> val_memo;
-    std::map<std::tuple<std::string, int, int>, std::string> shfl_memo;   // (var, lane offset, edge key)
+    // (var, lane offset, edge key, border constant): the constant is part of the
+    // key -- two CONSTANT-border consumers of the same row with different
+    // constants must not share an edge substitution
+    std::map<std::tuple<std::string, int, int, std::string>, std::string> shfl_memo;
     std::map<std::tuple<int, int, int>, SwReg> sw_memo;                     // SWAR values (image, slot, column)
     std::map<std::pair<int, int>, std::string> dl_memo;                      // delay-line rows read (image, age)
     std::string cur_it = "0";                                                // iteration index of the body being emitted
@@ -962,7 +965,7 @@ struct StreamGen {
         xe[img] = e;
     }
     std::string cvalx(const Op &op, int e) const { return f32 ? fconst(std::ldexp((double)(float)op.constant, -e)) : cval(op); }
-    std::map<std::tuple<std::string, int, int>, SwReg> swsh_memo;          // SWAR shuffles
+    std::map<std::tuple<std::string, int, int, long long>, SwReg> swsh_memo;   // SWAR shuffles (same key)
     // variant being emitted
     int dir = 1;
     bool el = false, er = false;
@@ -1063,7 +1066,7 @@ struct StreamGen {
         int idx = q - lo * V;
         const bool edge = (q < 0 && el) || (q >= V && er);
         const int ekey = edge ? op.mode * 64 + q : -1000;
-        auto key = std::make_tuple(row[idx], lo, ekey);
+        auto key = std::make_tuple(row[idx], lo, ekey, edge ? csub : std::string());
         auto it = shfl_memo.find(key);
         if (it != shfl_memo.end()) return it->second;
         std::string t = var();
@@ -1224,7 +1227,7 @@ struct StreamGen {
         int idx = q - lo * V;
         const bool edge = (q < 0 && el) || (q >= V && er);
         const int ekey = edge ? op.mode * 64 + q : -1000;
-        auto key = std::make_tuple(row[idx].lo, lo, ekey);
+        auto key = std::make_tuple(row[idx].lo, lo, ekey, edge ? csub : 0LL);
         auto it = swsh_memo.find(key);
         if (it != swsh_memo.end()) return it->second;
         SwReg t = row[idx];

@@ -154,6 +154,35 @@ def test_swar_constant_border_below_producer_range(width, opts):
     check(spec, got, O.run(spec, ins)[spec["outputs"][0]], f"constant_edge {width} {opts}")
 
 
+@pytest.mark.parametrize("dtype", ["f32", "u8x4"])
+@pytest.mark.parametrize("width", [512, 130])
+def test_two_constant_borders_on_one_row(dtype, width):
+    """Regression (fuzz seed 2031381): two CONSTANT-border local kernels with
+    different constants read the same producer row in one fused kernel.  The edge
+    lanes' substituted taps were memoised without the constant, so the second
+    kernel reused the first one's constant at the image's left and right columns
+    (normalised error 0.29 on the outer 3 columns)."""
+    p = P.Pipeline("two_constants", width, 64, dtype)
+    i = p.input()
+    mix = [[1, 0, 2], [0, 1, 0], [3, 0, 1]]            # rank > 1: taps read the producer row directly
+    if dtype == "f32":
+        a = p.local("a", i, [[0.25, 0.5, 0.25]], "mirror101")
+        b = p.local("b", a, [[v / 8.0 for v in r] for r in mix], "constant", constant=0.0)
+        c = p.local("c", a, [[v / 8.0 for v in r] for r in mix], "constant", constant=1.0)
+        p.output(p.point("d", [b, c], [P.L(0), P.L(1), P.SUB]))
+    else:
+        a = p.local("a", i, [[1, 2, 1]], "mirror101", post=[P.L(0), P.C(2), P.ADD, P.SHR(2), P.SAT])
+        b = p.local("b", a, mix, "constant", constant=0.0, post=[P.L(0), P.SHR(3), P.SAT])
+        c = p.local("c", a, mix, "constant", constant=255.0, post=[P.L(0), P.SHR(3), P.SAT])
+        p.output(p.point("d", [b, c], [P.L(0), P.L(1), P.SUB, P.C(255), P.ADD, P.SHR(1), P.SAT]))
+    spec = p.spec()
+    plan = make_plan(spec, "whole")
+    assert plan.num_launches == 1
+    ins = _inputs(spec, 5)
+    got = run_gpu(spec, plan, ins)[0]
+    check(spec, got, O.run(spec, ins)[spec["outputs"][0]], f"two_constants {dtype} {width}")
+
+
 def test_fig4_fused_on_gpu():
     """Fig. 4c through the fused GPU kernel: 763 at (0,0), 992 at (2,2)."""
     spec = P.fig4("clamp")

@@ -105,6 +105,22 @@ def jobs():
                          post=[P.L(0), P.C(16), P.ADD, P.SHR(5), P.C(0), P.ADD, P.SAT]))
         for o in (None, {"code_budget": 1000}):
             out.append((p.spec(), "b200", o, False))
+    for dtype in ("f32", "u8x4"):   # test_two_constant_borders_on_one_row
+        for width in (512, 130):
+            p = P.Pipeline("two_constants", width, 64, dtype)
+            i = p.input()
+            mix = [[1, 0, 2], [0, 1, 0], [3, 0, 1]]
+            if dtype == "f32":
+                a = p.local("a", i, [[0.25, 0.5, 0.25]], "mirror101")
+                b = p.local("b", a, [[v / 8.0 for v in r] for r in mix], "constant", constant=0.0)
+                c = p.local("c", a, [[v / 8.0 for v in r] for r in mix], "constant", constant=1.0)
+                p.output(p.point("d", [b, c], [P.L(0), P.L(1), P.SUB]))
+            else:
+                a = p.local("a", i, [[1, 2, 1]], "mirror101", post=[P.L(0), P.C(2), P.ADD, P.SHR(2), P.SAT])
+                b = p.local("b", a, mix, "constant", constant=0.0, post=[P.L(0), P.SHR(3), P.SAT])
+                c = p.local("c", a, mix, "constant", constant=255.0, post=[P.L(0), P.SHR(3), P.SAT])
+                p.output(p.point("d", [b, c], [P.L(0), P.L(1), P.SUB, P.C(255), P.ADD, P.SHR(1), P.SAT]))
+            out.append((p.spec(), "whole", None, False))
     out.append((P.deep10(260, 150), "b200", None, False))
     out.append((P.two_input(512, 300), "b200", None, False))
     out.append((P.harris(130, 97), "b200", None, False))
