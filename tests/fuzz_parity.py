@@ -129,7 +129,7 @@ def main():
         bad = bands_mode(cases)
         print(json.dumps({"mode": "bands", "dags": n, "seed0": seed0, "mismatches": len(bad), "bad": bad[:20]}))
         sys.exit(1 if bad else 0)
-    bad, worst, cancelled = [], 0.0, []
+    bad, worst, cancelled, ill = [], 0.0, [], []
     for spec, kind, opts, lab, seed in cases:
         ins = [gen.image(spec["dtype"], seed + 7 * j, spec["width"], spec["height"]) for j in range(spec["n_inputs"])]
         plan = make(spec, kind, opts, lab)
@@ -159,11 +159,31 @@ def main():
                     pw = float((d[sel] / a[sel]).max())
                     worst = max(worst, err)
                     ok = err <= 1e-5 and pw <= 1e-3
+            if not ok and spec["dtype"] == "f32" and kind != "unfused":
+                # f32 conditioning, not fusion: a random program (cancelling
+                # differences, ABS near zero) can exceed the pointwise bound in
+                # plain f32.  If the unfused GPU plan -- one kernel per operator,
+                # every intermediate materialised in f32 -- misses the oracle by as
+                # much, the fused result is as exact as f32 execution allows.
+                u = make(spec, "unfused", {}, None)
+                uo = [torch.empty(shape, dtype=dt, device="cuda") for _ in spec["outputs"]]
+                u.run(d_in, uo)
+                torch.cuda.synchronize()
+                ug = uo[spec["outputs"].index(img)].cpu().numpy()
+                ud = np.abs(ug.astype(np.float64) - r)
+                a = np.abs(r)
+                sel = a >= 1e-3 * a.max()
+                upw = float((ud[sel] / a[sel]).max()) if a.max() >= 1e-6 else 0.0
+                fpw = float((d[sel] / a[sel]).max()) if a.max() >= 1e-6 else 0.0
+                uerr = float(ud.max() / max(a.max(), 1e-30))
+                if upw > 1e-3 and fpw <= 4 * upw and float(d.max()) <= 4 * float(ud.max()) + 1e-12:
+                    ill.append({"seed": seed, "fused_pw": fpw, "unfused_pw": upw, "unfused_norm": uerr})
+                    ok = True
             if not ok:
                 bad.append({"seed": seed, "kind": kind, "opts": opts, "size": [spec["width"], spec["height"]],
                             "dtype": spec["dtype"], "ops": len(spec["ops"])})
     print(json.dumps({"dags": n, "seed0": seed0, "mismatches": len(bad), "worst_norm_err_f32": worst,
-                      "cancelled_outputs": len(cancelled), "bad": bad[:20]}))
+                      "cancelled_outputs": len(cancelled), "ill_conditioned_in_f32": ill[:20], "bad": bad[:20]}))
     sys.exit(1 if bad else 0)
 
 

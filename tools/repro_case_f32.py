@@ -35,9 +35,12 @@ for kk, o in [(kind, opts), (kind, {}), (kind, {"pdl": 0}), ("unfused", {}), ("b
         r = ref[img]
         d = np.abs(g - r)
         err = float(d.max() / max(np.abs(r).max(), 1e-30))
+        a = np.abs(r)
+        sel = a >= 1e-3 * a.max()
+        pw = float((d[sel] / a[sel]).max())
         bad = np.argwhere(d > 1e-4 * max(np.abs(r).max(), 1e-30))
         rows = sorted(set(bad[:, 0].tolist()))
         cols = sorted(set(bad[:, 1].tolist()))
-        rep.append({"img": img, "err": err, "n_bad": len(bad), "rows": rows[:12] + (["..."] if len(rows) > 12 else []),
+        rep.append({"img": img, "err": err, "pw": pw, "n_bad": len(bad), "rows": rows[:12] + (["..."] if len(rows) > 12 else []),
                     "cols": cols[:12] + (["..."] if len(cols) > 12 else []), "n_rows": len(rows), "n_cols": len(cols)})
     print(json.dumps({"plan": kk, "opts": o, "blocks": [list(b) for b in plan.blocks], "out": rep}), flush=True)
